@@ -1,0 +1,172 @@
+/*
+ * resccl.h — C ABI of the B200-native ResCCL hot path.
+ *
+ * ResCCL (Liu et al., SIGCOMM '25; PAPER.md line numbers cited as P:Lx-y) executes
+ * a collective-communication algorithm at primitive level: chunked send / recv /
+ * recvReduceCopy / recvReduceSend / recvCopySend steps that a host-side global
+ * scheduler (HPDS, Alg. 1) places on as few thread blocks as
+ * possible (state-based TB allocation, Eq. 7), run by lightweight
+ * generated kernels (§4.5).  Collective names: P:L436-438.
+ *
+ * Conventions (NCCL-like, implied by the paper's "relink and rebuild"
+ * integration):
+ *  - All pointers are plain device pointers (buffers) or host pointers (text,
+ *    handles, info).  No torch / C++ types cross this boundary.
+ *  - Counts are in elements.  AllGather's sendcount and ReduceScatter's recvcount
+ *    are per rank.  count == 0 is a successful no-op.
+ *  - In-place: AllReduce sendbuf == recvbuf; AllGather sendbuf == recvbuf +
+ *    rank*sendcount*size; ReduceScatter recvbuf == sendbuf + rank*recvcount*size.
+ *  - Collective calls only enqueue work on `stream` (cudaStream_t passed as void*;
+ *    NULL = legacy default stream); they never synchronise the device.
+ *  - All ranks issue the same collectives in the same order with the same count,
+ *    dtype and op; a communicator is not thread-safe.
+ *  - Every function returns a rescclResult_t; no exception crosses the ABI and the
+ *    library never aborts.  rescclGetLastError() returns a message for the last
+ *    failure on the calling thread.
+ *  - Ownership: the caller owns buffers and streams; a communicator owns its FIFO
+ *    arena, IPC mappings, compiled kernels and plans.  rescclLoadAlgorithm copies
+ *    the IR text; the rescclAlgo_t lives until rescclCommDestroy.
+ *
+ * Execution modes:
+ *  - Multi-process, one GPU per process (the production mode):
+ *    rescclCommCreate -> rescclCommGetHandle -> exchange the blobs (e.g. with
+ *    torch.distributed) -> rescclCommConnect; or rescclCommInit with an
+ *    allgather callback.  FIFOs are CUDA-IPC-mapped peer memory over NVLink.
+ *  - Single process (rescclCommInitAll): distinct devices use peer access; a
+ *    device listed several times hosts several "virtual ranks" whose buffers and
+ *    FIFOs share that GPU's HBM.  Virtual ranks of one device run as ONE kernel:
+ *    a collective is launched when the last virtual rank of the group has issued
+ *    it (on that caller's stream, ordered after the other callers' streams).
+ */
+#ifndef RESCCL_H_
+#define RESCCL_H_
+
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define RESCCL_VERSION 1000
+
+typedef struct rescclComm* rescclComm_t; /* opaque; owned by the library */
+typedef struct rescclAlgo* rescclAlgo_t; /* opaque; owned by its communicator */
+
+typedef enum {
+  rescclSuccess = 0,
+  rescclInvalidArgument = 1, /* null pointer, bad dtype/op/count, unsupported combination */
+  rescclInvalidUsage = 2,    /* IR rejected (malformed, conflicting, nranks mismatch, deadlocking
+                                plan), call order violated, arena exhausted */
+  rescclCudaError = 3,       /* CUDA runtime/driver or NVRTC failure */
+  rescclSystemError = 4,     /* IPC / OS failure */
+  rescclInternalError = 5,
+  rescclTimeout = 6          /* device watchdog fired (surfaced by rescclCommGetAsyncError) */
+} rescclResult_t;
+
+typedef enum { rescclInt32 = 0, rescclFloat32 = 1, rescclFloat16 = 2, rescclBfloat16 = 3 } rescclDataType_t;
+
+/* Sum is the paper's operator (AllReduce = ReduceScatter + AllGather);
+ * max/min are order-free extras. */
+typedef enum { rescclSum = 0, rescclMax = 1, rescclMin = 2 } rescclRedOp_t;
+
+typedef enum { rescclCollAllGather = 0, rescclCollReduceScatter = 1, rescclCollAllReduce = 2 } rescclColl_t;
+
+const char* rescclGetErrorString(rescclResult_t r);
+/* Message of the last failing call on this thread (static storage, never NULL). */
+const char* rescclGetLastError(void);
+int rescclGetVersion(void);
+
+/* ------------------------------------------------------------------ bootstrap */
+
+/* Create rank `rank` of an `nranks` communicator on device `cudaDev` (multi-process
+ * mode).  Allocates this rank's FIFO arena (RESCCL_ARENA_BYTES, default 128 MiB)
+ * in device memory.  Not usable until rescclCommConnect. */
+rescclResult_t rescclCommCreate(int rank, int nranks, int cudaDev, rescclComm_t* out);
+
+/* Write this rank's connection blob (CUDA IPC handle of the arena plus identity)
+ * into `buf`.  If buf is NULL, *len receives the required size; otherwise *len is
+ * the capacity on input and the written size on output. */
+rescclResult_t rescclCommGetHandle(rescclComm_t comm, void* buf, size_t* len);
+
+/* Map every peer's arena.  handles[k] / lens[k] is rank k's blob (as written by
+ * rescclCommGetHandle on rank k); handles[rank] is ignored. */
+rescclResult_t rescclCommConnect(rescclComm_t comm, const void* const* handles, const size_t* lens);
+
+/* Create + exchange + connect in one call.  `allgather` must gather `len` bytes
+ * from every rank into `out` (rank-major) and return 0 on success. */
+rescclResult_t rescclCommInit(rescclComm_t* out, int rank, int nranks, int cudaDev,
+                              int (*allgather)(const void* in, void* out, size_t len, void* ctx), void* ctx);
+
+/* Single-process communicators: comms[k] is rank k on device devlist[k].  Repeated
+ * devices host virtual ranks (see "Execution modes").  devlist == NULL means all
+ * ranks on device 0. */
+rescclResult_t rescclCommInitAll(rescclComm_t* comms, int ndev, const int* devlist);
+
+rescclResult_t rescclCommDestroy(rescclComm_t comm);
+rescclResult_t rescclCommRank(rescclComm_t comm, int* rank);
+rescclResult_t rescclCommCount(rescclComm_t comm, int* nranks);
+
+/* Device-side failures (watchdog timeout) recorded since the last call: *err is
+ * rescclSuccess or rescclTimeout.  Reads host-mapped memory; never blocks. */
+rescclResult_t rescclCommGetAsyncError(rescclComm_t comm, rescclResult_t* err);
+
+/* ------------------------------------------------------------------ algorithms */
+
+/* Parse, analyse, schedule and lower an algorithm (Parsing ->
+ * Analysis (DAG) -> Scheduling (HPDS) -> Lowering) and compile its kernel with NVRTC
+ * for sm_100a on first use.  irText (copied) is the one-transfer-per-line IR:
+ *     algo name=<s> coll=<allgather|reducescatter|allreduce> nranks=<N> nchunks=<N>
+ *          [nwarps=16] [instances=1] [chunkbytes=1048576] [fifodepth=4]
+ *          [linkmodel=pair|port] [fuse=1] [tbbudget=B]
+ *     t <src> <dst> <step> <chunk> <recv|rrc>
+ * Environment overrides: RESCCL_INSTANCES, RESCCL_CHUNK_BYTES, RESCCL_FIFO_DEPTH,
+ * RESCCL_NWARPS, RESCCL_LINK_MODEL, RESCCL_FUSE, RESCCL_TB_BUDGET.
+ * The loaded algorithm becomes the active one for its collective; with none
+ * loaded, the built-in ring is used.  All ranks must load the same algorithms in
+ * the same order.  InvalidUsage: nranks != communicator size, invalid IR (I6),
+ * same-step conflicts, deadlocking plan. */
+rescclResult_t rescclLoadAlgorithm(rescclComm_t comm, const char* irText, rescclAlgo_t* out);
+
+/* Make a previously loaded algorithm the active one for its collective. */
+rescclResult_t rescclSetActiveAlgorithm(rescclComm_t comm, rescclAlgo_t algo);
+
+/* JSON description of the lowered plan (Pr, per-rank CTAs/lanes/primitives,
+ * connection groups, TB counts, layout).  Same size protocol as rescclCommGetHandle. */
+rescclResult_t rescclGetPlanInfo(rescclAlgo_t algo, char* json, size_t* len);
+
+/* ------------------------------------------------------------------ collectives */
+
+/* out_r[i] = sum_k in_k[i].  sendbuf/recvbuf: count elements each. */
+rescclResult_t rescclAllReduce(const void* sendbuf, void* recvbuf, size_t count, rescclDataType_t dtype,
+                               rescclRedOp_t op, rescclComm_t comm, void* stream);
+/* out_r[k*sendcount + i] = in_k[i].  recvbuf: nranks*sendcount elements. */
+rescclResult_t rescclAllGather(const void* sendbuf, void* recvbuf, size_t sendcount, rescclDataType_t dtype,
+                               rescclComm_t comm, void* stream);
+/* out_r[i] = sum_k in_k[r*recvcount + i].  sendbuf: nranks*recvcount elements. */
+rescclResult_t rescclReduceScatter(const void* sendbuf, void* recvbuf, size_t recvcount,
+                                   rescclDataType_t dtype, rescclRedOp_t op, rescclComm_t comm, void* stream);
+
+/* ------------------------------------------------------------------ host-only tools (no GPU needed) */
+
+/* Built-in generators (name in ring|dbt|hm|synth; opts "g=4 seed=0 fanout=2").
+ * Writes IR text; size protocol as above. */
+rescclResult_t rescclGenerateIr(const char* name, rescclColl_t coll, int nranks, const char* opts, char* text,
+                                size_t* len);
+/* Plan an IR (header keys as for rescclLoadAlgorithm; `opts` overrides them) and
+ * write the plan JSON. */
+rescclResult_t rescclPlanIr(const char* irText, const char* opts, char* json, size_t* len);
+/* Generated CUDA source of an IR's kernel for ranks [rank_lo, rank_hi). */
+rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo, int rank_hi, char* src,
+                               size_t* len);
+/* NVRTC-compile the kernel of an IR for sm_100a (no GPU needed); *cubin_bytes
+ * receives the cubin size. */
+rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataType_t dtype, rescclRedOp_t op,
+                               size_t* cubin_bytes);
+/* Control-only blocking simulation of a planned IR (invariant I4): *ok = 1 if the
+ * plan completes for FIFO depth K and n_mb micro-batches. */
+rescclResult_t rescclCheckDeadlock(const char* irText, const char* opts, int K, int n_mb, int* ok);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RESCCL_H_ */

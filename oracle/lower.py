@@ -311,9 +311,10 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None) -> Plan:
         return out_prims, lanes
 
     out_prims, lanes = build(absorbed)
+    any_fused = bool(fuse) and any(absorbed[r] for r in range(N))
     plan = Plan(ir, model, edges, edge_rank, Pr, pidx, out_prims, lanes,
                 send_groups, recv_groups,
-                {r: len(act[r]) for r in range(N)}, bool(fuse))
+                {r: len(act[r]) for r in range(N)}, any_fused)
     plan._act = act
     if fuse and any(absorbed[r] for r in range(N)):
         from .replay import deadlock_free

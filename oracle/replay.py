@@ -444,3 +444,31 @@ def check_plan(plan: Plan) -> None:
                     acc |= a
         sb, rb = plan.clique_bound(r)
         assert len(plan.send_groups[r]) >= sb and len(plan.recv_groups[r]) >= rb
+
+
+# ------------------------------------------------------------------ step-order dataflow (sampled)
+
+def dataflow_values(ir, chunk_inputs, dtype: str, op: str = "sum"):
+    """The IR executed literally in step order on per-chunk value vectors.
+
+    ``chunk_inputs[r][c]`` is rank r's input restricted to any set of element
+    positions of chunk c (the same positions for every rank); returns
+    ``out[r][c]`` at those positions.  Because every element of a chunk follows
+    the same transfers, this gives the schedule's exact result (same association
+    order as ``replay``, R8) for sampled elements of arbitrarily large buffers.
+    Locations never written keep their input (AG: owner's chunk only is defined)."""
+    N = ir.nranks
+    val = {}
+    for r in range(N):
+        for c in range(ir.nchunks):
+            if ir.coll == "allgather":
+                val[(r, c)] = chunk_inputs[r][c] if r == c else None
+            else:
+                val[(r, c)] = chunk_inputs[r][c]
+    for t in sorted(ir.transfers, key=lambda t: t.step):
+        incoming = val[(t.src, t.chunk)]
+        if t.op == "recv":
+            val[(t.dst, t.chunk)] = incoming.copy()
+        else:
+            val[(t.dst, t.chunk)] = combine(val[(t.dst, t.chunk)], incoming, dtype, op)
+    return [[val[(r, c)] for c in range(ir.nchunks)] for r in range(N)]

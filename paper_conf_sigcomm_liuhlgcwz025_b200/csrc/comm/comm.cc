@@ -1,0 +1,1032 @@
+// ResCCL control plane + C ABI (include/resccl.h).
+//
+// The paper's middle layer is "CPU-side coordination and management for the runtime"
+// (P:L2030-2035).  Here it owns: communicators and their FIFO arenas, CUDA-IPC
+// mapping of peer arenas (NVLink peer memory), loading algorithms (parse -> DAG ->
+// HPDS -> lower), NVRTC compilation of the generated kernel for
+// sm_100a (cached per plan/dtype/op), per-call geometry and the launch.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <nvrtc.h>
+
+#include <unistd.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <deque>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "../../../include/resccl.h"
+#include "../plan/codegen.h"
+#include "../plan/ir.h"
+#include "../plan/plan.h"
+
+static const char* kDeviceSrc =
+#include "device_src.inc"
+    ;
+
+namespace {
+
+using namespace resccl;
+constexpr int kMaxR = 32;
+
+// host mirror of rdev::KArgs (resccl_device.cuh)
+struct KArgs {
+  char* arena[kMaxR];
+  const char* sendbuf[kMaxR];
+  char* recvbuf[kMaxR];
+  char* scratch[kMaxR];
+  unsigned long long mb_base;
+  long long count, C, M, Mi;
+  int n_mb;
+  int block_base;
+  int* err;
+  unsigned long long timeout_ns;
+};
+
+thread_local std::string g_last_error;
+
+struct Error {
+  rescclResult_t code;
+  std::string msg;
+};
+
+[[noreturn]] void fail(rescclResult_t c, const std::string& m) { throw Error{c, m}; }
+
+void cuda_check(cudaError_t e, const char* what) {
+  if (e != cudaSuccess) fail(rescclCudaError, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+// ---------------------------------------------------------------- driver entry points (no libcuda link)
+struct Driver {
+  CUresult (*ModuleLoadData)(CUmodule*, const void*) = nullptr;
+  CUresult (*ModuleGetFunction)(CUfunction*, CUmodule, const char*) = nullptr;
+  CUresult (*ModuleUnload)(CUmodule) = nullptr;
+  CUresult (*LaunchCooperativeKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                                      unsigned, CUstream, void**) = nullptr;
+  CUresult (*LaunchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                           CUstream, void**, void**) = nullptr;
+  CUresult (*GetErrorString)(CUresult, const char**) = nullptr;
+  bool ok = false;
+};
+
+template <class F>
+void entry(const char* name, F* fn) {
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  cuda_check(cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q), name);
+  if (q != cudaDriverEntryPointSuccess || !p) fail(rescclCudaError, std::string("driver entry point ") + name);
+  *fn = (F)p;
+}
+
+Driver& driver() {
+  static Driver d;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    try {
+      entry("cuModuleLoadData", &d.ModuleLoadData);
+      entry("cuModuleGetFunction", &d.ModuleGetFunction);
+      entry("cuModuleUnload", &d.ModuleUnload);
+      entry("cuLaunchCooperativeKernel", &d.LaunchCooperativeKernel);
+      entry("cuLaunchKernel", &d.LaunchKernel);
+      entry("cuGetErrorString", &d.GetErrorString);
+      d.ok = true;
+    } catch (Error&) {
+      d.ok = false;
+    }
+  });
+  if (!d.ok) fail(rescclCudaError, "CUDA driver entry points unavailable (no GPU / driver?)");
+  return d;
+}
+
+void cu_check(CUresult r, const char* what) {
+  if (r != CUDA_SUCCESS) {
+    const char* s = "?";
+    if (driver().GetErrorString) driver().GetErrorString(r, &s);
+    fail(rescclCudaError, std::string(what) + ": " + s);
+  }
+}
+
+// ---------------------------------------------------------------- options
+struct Options {
+  int instances = 1;
+  int64_t chunk_bytes = 1 << 20;  // Table 2
+  int fifo_depth = 4;
+  int nwarps = 16;                // Table 2
+  LinkModel model = LinkModel::Pair;
+  bool fuse = true;
+  int tb_budget = 0;
+};
+
+std::map<std::string, std::string> parse_kv(const char* s) {
+  std::map<std::string, std::string> kv;
+  if (!s) return kv;
+  std::istringstream is(s);
+  std::string w;
+  while (is >> w) {
+    auto e = w.find('=');
+    if (e == std::string::npos) fail(rescclInvalidArgument, "option '" + w + "' is not key=value");
+    kv[w.substr(0, e)] = w.substr(e + 1);
+  }
+  return kv;
+}
+
+long to_long(const std::string& v, const std::string& k) {
+  try {
+    size_t p = 0;
+    long x = std::stol(v, &p);
+    if (p != v.size()) throw 0;
+    return x;
+  } catch (...) {
+    fail(rescclInvalidArgument, "option " + k + " is not an integer: " + v);
+  }
+}
+
+void apply_kv(Options& o, const std::string& k, const std::string& v) {
+  if (k == "instances") o.instances = (int)to_long(v, k);
+  else if (k == "chunkbytes") o.chunk_bytes = to_long(v, k);
+  else if (k == "fifodepth") o.fifo_depth = (int)to_long(v, k);
+  else if (k == "nwarps") o.nwarps = (int)to_long(v, k);
+  else if (k == "fuse") o.fuse = to_long(v, k) != 0;
+  else if (k == "tbbudget") o.tb_budget = (int)to_long(v, k);
+  else if (k == "linkmodel") {
+    if (v == "pair") o.model = LinkModel::Pair;
+    else if (v == "port") o.model = LinkModel::Port;
+    else fail(rescclInvalidArgument, "linkmodel must be pair|port");
+  }
+}
+
+Options make_options(const Ir& ir, const char* extra) {
+  Options o;
+  o.nwarps = ir.nwarps;
+  for (auto& kv : ir.extra) apply_kv(o, kv.first, kv.second);
+  static const std::pair<const char*, const char*> envs[] = {
+      {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
+      {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
+      {"RESCCL_TB_BUDGET", "tbbudget"}};
+  for (auto& e : envs)
+    if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
+  for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
+  if (o.instances < 1 || o.instances > 64) fail(rescclInvalidArgument, "instances must be 1..64");
+  if (o.fifo_depth < 1 || o.fifo_depth > 64) fail(rescclInvalidArgument, "fifodepth must be 1..64");
+  if (o.chunk_bytes < 256 || o.chunk_bytes > (1ll << 30)) fail(rescclInvalidArgument, "chunkbytes out of range");
+  if (o.nwarps < 2 || o.nwarps > 32 || o.nwarps % 2) fail(rescclInvalidArgument, "nwarps must be even, 2..32");
+  return o;
+}
+
+// Plan an IR under the options.  A TB budget B picks the link
+// model and the instance count: instances = floor(B / T_min) under the pair model;
+// below T_min the port model (one duplex CTA per rank) with B instances.
+Plan make_plan(const Ir& ir, Options& o) {
+  if (o.tb_budget > 0) {
+    Plan p = lower(ir, LinkModel::Pair, o.fuse);
+    int tmin = 1;
+    for (auto& r : p.ranks) tmin = std::max(tmin, (int)r.ctas.size());
+    if (o.tb_budget >= tmin) {
+      o.model = LinkModel::Pair;
+      o.instances = std::max(1, o.tb_budget / tmin);
+      return p;
+    }
+    o.model = LinkModel::Port;
+    Plan q = lower(ir, LinkModel::Port, o.fuse);
+    int t1 = 1;
+    for (auto& r : q.ranks) t1 = std::max(t1, (int)r.ctas.size());
+    o.instances = std::max(1, o.tb_budget / t1);
+    return q;
+  }
+  return lower(ir, o.model, o.fuse);
+}
+
+Plan plan_checked(const Ir& ir, Options& o) {
+  Plan p = make_plan(ir, o);
+  std::string why;
+  for (int nmb : {1, 2, 3})
+    if (!deadlock_free(p, 1, nmb, &why)) fail(rescclInvalidUsage, "plan deadlocks: " + why);
+  return p;
+}
+
+int elt_size(rescclDataType_t t) {
+  switch (t) {
+    case rescclInt32: case rescclFloat32: return 4;
+    case rescclFloat16: case rescclBfloat16: return 2;
+  }
+  return 0;
+}
+const char* dtype_tag(rescclDataType_t t) {
+  switch (t) {
+    case rescclInt32: return "rdev::TI32";
+    case rescclFloat32: return "rdev::TF32";
+    case rescclFloat16: return "rdev::TF16";
+    case rescclBfloat16: return "rdev::TBF16";
+  }
+  return "?";
+}
+
+// ---------------------------------------------------------------- NVRTC
+std::vector<char> nvrtc_compile(const std::string& gen_src, rescclDataType_t dt, rescclRedOp_t op, bool gpu_scope,
+                                std::string* log_out = nullptr) {
+  const char* hdrs[] = {kDeviceSrc};
+  const char* hdr_names[] = {"resccl_device.cuh"};
+  nvrtcProgram prog;
+  if (nvrtcCreateProgram(&prog, gen_src.c_str(), "resccl_gen.cu", 1, hdrs, hdr_names) != NVRTC_SUCCESS)
+    fail(rescclCudaError, "nvrtcCreateProgram failed");
+  std::string dT = std::string("-DRESCCL_T=") + dtype_tag(dt);
+  std::string dO = "-DRESCCL_OP=" + std::to_string((int)op);
+  std::vector<const char*> opts = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", dT.c_str(), dO.c_str(),
+                                   "-DRESCCL_MAXR=32"};
+  nvrtcResult rc = nvrtcCompileProgram(prog, (int)opts.size(), opts.data());
+  size_t logsz = 0;
+  nvrtcGetProgramLogSize(prog, &logsz);
+  std::string log(logsz, '\0');
+  if (logsz) nvrtcGetProgramLog(prog, &log[0]);
+  if (log_out) *log_out = log;
+  if (rc != NVRTC_SUCCESS) {
+    nvrtcDestroyProgram(&prog);
+    fail(rescclCudaError, std::string("NVRTC: ") + nvrtcGetErrorString(rc) + "\n" + log.substr(0, 4000));
+  }
+  size_t n = 0;
+  nvrtcGetCUBINSize(prog, &n);
+  std::vector<char> cubin(n);
+  nvrtcGetCUBIN(prog, cubin.data());
+  nvrtcDestroyProgram(&prog);
+  return cubin;
+}
+
+// ---------------------------------------------------------------- algorithm state
+struct Kern {
+  CUmodule mod = nullptr;
+  CUfunction fn = nullptr;
+};
+
+struct AlgoShared {
+  std::string text;
+  Ir ir;
+  Options opt;
+  Plan plan;
+  Layout lay;
+  std::string json;
+  unsigned long long mb_cum = 0;       // virtual group: one counter for all ranks
+  std::map<std::string, Kern> kernels;  // key: dtype/op/ranks/scope
+  std::vector<char*> region;           // virtual group: per-rank plan region (one allocation)
+  char* region_alloc = nullptr;
+  int64_t region_off = 0;              // multi-process: offset inside the arena
+};
+
+}  // namespace
+
+struct rescclAlgo {
+  std::shared_ptr<AlgoShared> s;
+  rescclComm* comm = nullptr;
+  unsigned long long mb_cum = 0;  // multi-process: this rank's counter
+};
+
+namespace {
+struct Group;
+}
+
+struct rescclComm {
+  int rank = 0, nranks = 1, dev = 0;
+  bool connected = false;
+  int mode = 0;  // 0 multi-process (IPC), 1 virtual (shared device), 2 single-process multi-device
+  Group* group = nullptr;
+  char* arena = nullptr;
+  size_t arena_bytes = 0, arena_used = 0;
+  std::vector<char*> peer_arena;  // size nranks (self = arena)
+  std::vector<bool> peer_opened;
+  int* err_host = nullptr;
+  int* err_dev = nullptr;
+  std::vector<std::unique_ptr<rescclAlgo>> algos;
+  rescclAlgo* active[3] = {nullptr, nullptr, nullptr};
+  char* scratch = nullptr;
+  size_t scratch_bytes = 0;
+  std::vector<rescclComm*> peers_local;  // mode 2: every comm of the process
+};
+
+namespace {
+
+struct Pending {
+  int coll;
+  size_t count;
+  int dtype, op;
+  int arrived = 0;
+  AlgoShared* algo = nullptr;
+  std::vector<const void*> send;
+  std::vector<void*> recv;
+  std::vector<cudaStream_t> streams;
+};
+
+struct Group {
+  int dev = 0, nranks = 0;
+  std::vector<rescclComm*> comms;
+  std::map<std::string, std::shared_ptr<AlgoShared>> algos;  // by IR text + opts
+  std::vector<unsigned long long> issued;                   // per rank: collectives issued
+  std::deque<Pending> pending;                               // pending[0] = sequence `base`
+  unsigned long long base = 0;
+  int* err_host = nullptr;
+  int* err_dev = nullptr;
+  std::vector<cudaEvent_t> events;
+  int refs = 0;
+};
+
+unsigned long long timeout_ns() {
+  const char* v = getenv("RESCCL_TIMEOUT_MS");
+  long ms = v ? atol(v) : 30000;
+  if (ms <= 0) ms = 30000;
+  return (unsigned long long)ms * 1000000ull;
+}
+
+size_t arena_default() {
+  const char* v = getenv("RESCCL_ARENA_BYTES");
+  return v ? (size_t)atoll(v) : (size_t)128 << 20;
+}
+
+std::shared_ptr<AlgoShared> build_algo(const std::string& text, int nranks) {
+  auto a = std::make_shared<AlgoShared>();
+  a->text = text;
+  try {
+    a->ir = parse_ir(text);
+  } catch (PlanError& e) {
+    fail(rescclInvalidUsage, std::string("IR: ") + e.what());
+  }
+  if (a->ir.nranks != nranks)
+    fail(rescclInvalidUsage, "IR nranks=" + std::to_string(a->ir.nranks) + " != communicator size " +
+                                 std::to_string(nranks));
+  if (nranks > kMaxR) fail(rescclInvalidUsage, "at most 32 ranks per communicator");
+  try {
+    a->opt = make_options(a->ir, nullptr);
+    a->plan = plan_checked(a->ir, a->opt);
+    a->lay = make_layout(a->plan, a->opt.fifo_depth, a->opt.instances, a->opt.chunk_bytes);
+  } catch (PlanError& e) {
+    fail(rescclInvalidUsage, std::string("plan: ") + e.what());
+  }
+  return a;
+}
+
+std::string info_json(const AlgoShared& a) {
+  std::ostringstream o;
+  std::string pj = plan_json(a.plan);
+  o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
+    << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"linkmodel\":\""
+    << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
+    << ",\"ctas\":[";
+  for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];
+  o << "],\"blocks_per_rank\":[";
+  for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r] * a.opt.instances;
+  o << "]}";
+  return o.str();
+}
+
+Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, int hi, bool gpu_scope) {
+  std::string key = std::to_string((int)dt) + "/" + std::to_string((int)op) + "/" + std::to_string(lo) + "-" +
+                    std::to_string(hi) + "/" + (gpu_scope ? "g" : "s");
+  auto it = a.kernels.find(key);
+  if (it != a.kernels.end()) return it->second;
+  CodegenOpts co;
+  co.rank_lo = lo;
+  co.rank_hi = hi;
+  co.gpu_scope = gpu_scope;
+  co.nwarps = a.opt.nwarps;
+  std::string src = codegen(a.plan, a.lay, co);
+  std::vector<char> cubin = nvrtc_compile(src, dt, op, gpu_scope);
+  Kern k;
+  cu_check(driver().ModuleLoadData(&k.mod, cubin.data()), "cuModuleLoadData");
+  cu_check(driver().ModuleGetFunction(&k.fn, k.mod, "resccl_kernel"), "cuModuleGetFunction");
+  return a.kernels[key] = k;
+}
+
+void set_err(const Error& e) { g_last_error = e.msg; }
+
+#define API_BEGIN try {
+#define API_END                                      \
+  }                                                  \
+  catch (Error & e) {                                \
+    set_err(e);                                      \
+    return e.code;                                   \
+  }                                                  \
+  catch (PlanError & e) {                            \
+    g_last_error = e.what();                         \
+    return rescclInvalidUsage;                       \
+  }                                                  \
+  catch (std::exception & e) {                       \
+    g_last_error = e.what();                         \
+    return rescclInternalError;                      \
+  }                                                  \
+  catch (...) {                                      \
+    g_last_error = "unknown exception";              \
+    return rescclInternalError;                      \
+  }                                                  \
+  return rescclSuccess;
+
+void write_out(const std::string& s, void* buf, size_t* len) {
+  if (!len) fail(rescclInvalidArgument, "len is NULL");
+  if (!buf) {
+    *len = s.size() + 1;
+    return;
+  }
+  if (*len < s.size() + 1) {
+    size_t need = s.size() + 1;
+    *len = need;
+    fail(rescclInvalidArgument, "buffer too small (need " + std::to_string(need) + " bytes)");
+  }
+  memcpy(buf, s.c_str(), s.size() + 1);
+  *len = s.size() + 1;
+}
+
+void alloc_err_word(int** host, int** dev) {
+  cuda_check(cudaHostAlloc((void**)host, 64, cudaHostAllocMapped | cudaHostAllocPortable), "cudaHostAlloc");
+  memset(*host, 0, 64);
+  cuda_check(cudaHostGetDevicePointer((void**)dev, *host, 0), "cudaHostGetDevicePointer");
+}
+
+// ---------------------------------------------------------------- launching
+struct CallDesc {
+  int coll;
+  size_t count;
+  rescclDataType_t dt;
+  rescclRedOp_t op;
+};
+
+Geometry call_geometry(const AlgoShared& a, const CallDesc& c) {
+  return geometry(a.ir.coll, a.ir.nranks, (int64_t)c.count, elt_size(c.dt), a.opt.chunk_bytes, a.opt.instances);
+}
+
+void ensure_scratch(rescclComm* comm, size_t bytes) {
+  if (comm->scratch_bytes >= bytes) return;
+  cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+  char* p = nullptr;
+  cuda_check(cudaMalloc((void**)&p, bytes), "cudaMalloc(scratch)");
+  // the old buffer may still be in use by queued kernels: keep it until destroy
+  if (comm->scratch) {
+    static std::vector<char*> graveyard;
+    graveyard.push_back(comm->scratch);
+  }
+  comm->scratch = p;
+  comm->scratch_bytes = bytes;
+}
+
+void launch(Kern& k, int grid, int block, KArgs& args, cudaStream_t s) {
+  void* params[] = {&args};
+  cu_check(driver().LaunchCooperativeKernel(k.fn, grid, 1, 1, block, 1, 1, 0, (CUstream)s, params),
+           "cuLaunchCooperativeKernel");
+}
+
+void fill_geometry(KArgs& ka, const Geometry& g, size_t count) {
+  ka.count = (long long)count;
+  ka.C = g.C;
+  ka.M = g.M;
+  ka.Mi = g.Mi;
+  ka.n_mb = g.n_mb;
+}
+
+// multi-process / multi-device path: this rank alone
+void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const void* send, void* recv,
+                 cudaStream_t s) {
+  AlgoShared& a = *algo->s;
+  Geometry g = call_geometry(a, c);
+  if (g.n_mb == 0) return;
+  cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+  KArgs ka;
+  memset(&ka, 0, sizeof(ka));
+  for (int q = 0; q < comm->nranks; ++q) ka.arena[q] = comm->peer_arena[q] + a.region_off;
+  ka.sendbuf[comm->rank] = (const char*)send;
+  ka.recvbuf[comm->rank] = (char*)recv;
+  if (a.ir.coll == Coll::ReduceScatter) {
+    ensure_scratch(comm, c.count * comm->nranks * elt_size(c.dt));
+    ka.scratch[comm->rank] = comm->scratch;
+  }
+  fill_geometry(ka, g, c.count);
+  ka.mb_base = algo->mb_cum;
+  ka.block_base = a.lay.pair_start[comm->rank] * a.opt.instances;
+  ka.err = comm->err_dev;
+  ka.timeout_ns = timeout_ns();
+  Kern& k = get_kernel(a, c.dt, c.op, comm->rank, comm->rank + 1, false);
+  launch(k, a.lay.ctas[comm->rank] * a.opt.instances, 32 * a.opt.nwarps, ka, s);
+  algo->mb_cum += (unsigned long long)g.n_mb;
+}
+
+// virtual group: all ranks in one kernel, when the last rank arrives
+void group_launch(Group* G, Pending& p) {
+  AlgoShared& a = *p.algo;
+  CallDesc c{p.coll, p.count, (rescclDataType_t)p.dtype, (rescclRedOp_t)p.op};
+  Geometry g = call_geometry(a, c);
+  if (g.n_mb == 0) return;
+  cuda_check(cudaSetDevice(G->dev), "cudaSetDevice");
+  KArgs ka;
+  memset(&ka, 0, sizeof(ka));
+  for (int q = 0; q < G->nranks; ++q) {
+    ka.arena[q] = a.region[q];
+    ka.sendbuf[q] = (const char*)p.send[q];
+    ka.recvbuf[q] = (char*)p.recv[q];
+    if (a.ir.coll == Coll::ReduceScatter) {
+      ensure_scratch(G->comms[q], c.count * G->nranks * elt_size(c.dt));
+      ka.scratch[q] = G->comms[q]->scratch;
+    }
+  }
+  fill_geometry(ka, g, c.count);
+  ka.mb_base = a.mb_cum;
+  ka.block_base = 0;
+  ka.err = G->err_dev;
+  ka.timeout_ns = timeout_ns();
+  Kern& k = get_kernel(a, c.dt, c.op, 0, G->nranks, true);
+  cudaStream_t ls = p.streams.back();
+  // order the launch after every caller's stream, and every caller's stream after it
+  std::vector<cudaStream_t> others;
+  for (auto s : p.streams)
+    if (s != ls && std::find(others.begin(), others.end(), s) == others.end()) others.push_back(s);
+  while (G->events.size() < 2 * others.size() + 1) {
+    cudaEvent_t e;
+    cuda_check(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
+    G->events.push_back(e);
+  }
+  for (size_t i = 0; i < others.size(); ++i) {
+    cuda_check(cudaEventRecord(G->events[i], others[i]), "cudaEventRecord");
+    cuda_check(cudaStreamWaitEvent(ls, G->events[i], 0), "cudaStreamWaitEvent");
+  }
+  launch(k, a.lay.total_pairs * a.opt.instances, 32 * a.opt.nwarps, ka, ls);
+  a.mb_cum += (unsigned long long)g.n_mb;
+  if (!others.empty()) {
+    cudaEvent_t done = G->events[others.size()];
+    cuda_check(cudaEventRecord(done, ls), "cudaEventRecord");
+    for (auto s : others) cuda_check(cudaStreamWaitEvent(s, done, 0), "cudaStreamWaitEvent");
+  }
+}
+
+rescclAlgo* ensure_algo(rescclComm* comm, Coll coll);
+
+void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t count, rescclDataType_t dt,
+                rescclRedOp_t op, void* stream) {
+  if (!comm) fail(rescclInvalidArgument, "comm is NULL");
+  if (!comm->connected) fail(rescclInvalidUsage, "communicator not connected");
+  if (elt_size(dt) == 0) fail(rescclInvalidArgument, "bad dtype");
+  if ((int)op < 0 || (int)op > 2) fail(rescclInvalidArgument, "bad op");
+  if (count > 0 && (!send || !recv)) fail(rescclInvalidArgument, "null buffer");
+  rescclAlgo* algo = ensure_algo(comm, (Coll)coll);
+  cudaStream_t s = (cudaStream_t)stream;
+  if (comm->mode != 1) {
+    if (count == 0) return;
+    launch_rank(comm, algo, CallDesc{coll, count, dt, op}, send, recv, s);
+    return;
+  }
+  Group* G = comm->group;
+  unsigned long long seq = G->issued[comm->rank]++;
+  if (seq < G->base) fail(rescclInternalError, "group sequence underflow");
+  while (G->pending.size() <= seq - G->base) G->pending.emplace_back();
+  Pending& p = G->pending[seq - G->base];
+  if (p.arrived == 0) {
+    p.coll = coll;
+    p.count = count;
+    p.dtype = (int)dt;
+    p.op = (int)op;
+    p.algo = algo->s.get();
+    p.send.assign(G->nranks, nullptr);
+    p.recv.assign(G->nranks, nullptr);
+  } else if (p.coll != coll || p.count != count || p.dtype != (int)dt || p.op != (int)op ||
+             p.algo != algo->s.get()) {
+    G->issued[comm->rank]--;
+    fail(rescclInvalidUsage, "virtual ranks issued mismatching collectives");
+  }
+  p.send[comm->rank] = send;
+  p.recv[comm->rank] = recv;
+  p.streams.push_back(s);
+  p.arrived++;
+  while (!G->pending.empty() && G->pending.front().arrived == G->nranks) {
+    Pending q = G->pending.front();
+    G->pending.pop_front();
+    G->base++;
+    if (q.count > 0) group_launch(G, q);
+  }
+}
+
+// ---------------------------------------------------------------- algorithm loading
+rescclAlgo* load_algo(rescclComm* comm, const std::string& text) {
+  std::shared_ptr<AlgoShared> s;
+  if (comm->mode == 1) {
+    Group* G = comm->group;
+    auto it = G->algos.find(text);
+    if (it != G->algos.end()) {
+      s = it->second;
+    } else {
+      s = build_algo(text, comm->nranks);
+      cuda_check(cudaSetDevice(G->dev), "cudaSetDevice");
+      size_t bytes = (size_t)s->lay.region_bytes * G->nranks;
+      cuda_check(cudaMalloc((void**)&s->region_alloc, bytes), "cudaMalloc(region)");
+      cuda_check(cudaMemset(s->region_alloc, 0, bytes), "cudaMemset(region)");
+      cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
+      for (int q = 0; q < G->nranks; ++q) s->region.push_back(s->region_alloc + (size_t)q * s->lay.region_bytes);
+      G->algos[text] = s;
+    }
+  } else {
+    s = build_algo(text, comm->nranks);
+    size_t need = (size_t)s->lay.region_bytes;
+    if (comm->arena_used + need > comm->arena_bytes)
+      fail(rescclInvalidUsage, "FIFO arena exhausted: need " + std::to_string(comm->arena_used + need) +
+                                   " bytes; raise RESCCL_ARENA_BYTES");
+    s->region_off = (int64_t)comm->arena_used;
+    comm->arena_used += (need + 4095) / 4096 * 4096;
+  }
+  auto algo = std::make_unique<rescclAlgo>();
+  algo->s = s;
+  algo->comm = comm;
+  rescclAlgo* raw = algo.get();
+  comm->algos.push_back(std::move(algo));
+  comm->active[(int)s->ir.coll] = raw;
+  return raw;
+}
+
+rescclAlgo* ensure_algo(rescclComm* comm, Coll coll) {
+  rescclAlgo* a = comm->active[(int)coll];
+  if (a) return a;
+  Ir ir = gen_ring(coll, comm->nranks);
+  return load_algo(comm, ir.to_text());
+}
+
+Group* make_group(int dev, int n) {
+  Group* G = new Group();
+  G->dev = dev;
+  G->nranks = n;
+  G->issued.assign(n, 0);
+  cuda_check(cudaSetDevice(dev), "cudaSetDevice");
+  alloc_err_word(&G->err_host, &G->err_dev);
+  return G;
+}
+
+Plan plan_from(const char* irText, const char* opts, Options* o_out, Ir* ir_out) {
+  if (!irText) fail(rescclInvalidArgument, "irText is NULL");
+  Ir ir = parse_ir(irText);
+  Options o = make_options(ir, opts);
+  Plan p = make_plan(ir, o);
+  if (o_out) *o_out = o;
+  if (ir_out) *ir_out = ir;
+  return p;
+}
+
+}  // namespace
+
+// =================================================================== C ABI
+extern "C" {
+
+const char* rescclGetErrorString(rescclResult_t r) {
+  switch (r) {
+    case rescclSuccess: return "success";
+    case rescclInvalidArgument: return "invalid argument";
+    case rescclInvalidUsage: return "invalid usage";
+    case rescclCudaError: return "CUDA error";
+    case rescclSystemError: return "system error";
+    case rescclInternalError: return "internal error";
+    case rescclTimeout: return "timeout (device watchdog)";
+  }
+  return "unknown result";
+}
+
+const char* rescclGetLastError(void) { return g_last_error.c_str(); }
+int rescclGetVersion(void) { return RESCCL_VERSION; }
+
+struct Blob {
+  unsigned magic;
+  int rank, nranks, dev;
+  unsigned long long arena_bytes;
+  cudaIpcMemHandle_t handle;
+  int pid;
+};
+
+rescclResult_t rescclCommCreate(int rank, int nranks, int cudaDev, rescclComm_t* out) {
+  API_BEGIN
+  if (!out) fail(rescclInvalidArgument, "out is NULL");
+  if (nranks < 1 || nranks > kMaxR || rank < 0 || rank >= nranks) fail(rescclInvalidArgument, "bad rank/nranks");
+  auto c = std::make_unique<rescclComm>();
+  c->rank = rank;
+  c->nranks = nranks;
+  c->dev = cudaDev;
+  c->mode = 0;
+  cuda_check(cudaSetDevice(cudaDev), "cudaSetDevice");
+  c->arena_bytes = arena_default();
+  cuda_check(cudaMalloc((void**)&c->arena, c->arena_bytes), "cudaMalloc(arena)");
+  cuda_check(cudaMemset(c->arena, 0, c->arena_bytes), "cudaMemset(arena)");
+  cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
+  alloc_err_word(&c->err_host, &c->err_dev);
+  c->peer_arena.assign(nranks, nullptr);
+  c->peer_opened.assign(nranks, false);
+  c->peer_arena[rank] = c->arena;
+  *out = c.release();
+  API_END
+}
+
+rescclResult_t rescclCommGetHandle(rescclComm_t comm, void* buf, size_t* len) {
+  API_BEGIN
+  if (!comm || !len) fail(rescclInvalidArgument, "null argument");
+  if (comm->mode != 0) fail(rescclInvalidUsage, "handles exist only in multi-process mode");
+  if (!buf) {
+    *len = sizeof(Blob);
+    return rescclSuccess;
+  }
+  if (*len < sizeof(Blob)) fail(rescclInvalidArgument, "handle buffer too small");
+  Blob b;
+  memset(&b, 0, sizeof(b));
+  b.magic = 0x52435343u;
+  b.rank = comm->rank;
+  b.nranks = comm->nranks;
+  b.dev = comm->dev;
+  b.arena_bytes = comm->arena_bytes;
+  b.pid = (int)getpid();
+  cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+  cuda_check(cudaIpcGetMemHandle(&b.handle, comm->arena), "cudaIpcGetMemHandle");
+  memcpy(buf, &b, sizeof(b));
+  *len = sizeof(Blob);
+  API_END
+}
+
+rescclResult_t rescclCommConnect(rescclComm_t comm, const void* const* handles, const size_t* lens) {
+  API_BEGIN
+  if (!comm || !handles || !lens) fail(rescclInvalidArgument, "null argument");
+  if (comm->mode != 0) fail(rescclInvalidUsage, "connect is for multi-process communicators");
+  cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+  for (int q = 0; q < comm->nranks; ++q) {
+    if (q == comm->rank) continue;
+    if (!handles[q] || lens[q] < sizeof(Blob)) fail(rescclInvalidArgument, "bad handle blob");
+    Blob b;
+    memcpy(&b, handles[q], sizeof(b));
+    if (b.magic != 0x52435343u || b.rank != q || b.nranks != comm->nranks)
+      fail(rescclInvalidArgument, "handle blob of rank " + std::to_string(q) + " is inconsistent");
+    if (b.arena_bytes != comm->arena_bytes) fail(rescclInvalidUsage, "ranks use different RESCCL_ARENA_BYTES");
+    void* p = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&p, b.handle, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess)
+      fail(rescclSystemError, "cudaIpcOpenMemHandle(rank " + std::to_string(q) + "): " + cudaGetErrorString(e));
+    comm->peer_arena[q] = (char*)p;
+    comm->peer_opened[q] = true;
+  }
+  comm->connected = true;
+  API_END
+}
+
+rescclResult_t rescclCommInit(rescclComm_t* out, int rank, int nranks, int cudaDev,
+                              int (*allgather)(const void*, void*, size_t, void*), void* ctx) {
+  API_BEGIN
+  if (!out || !allgather) fail(rescclInvalidArgument, "null argument");
+  rescclComm_t c = nullptr;
+  rescclResult_t r = rescclCommCreate(rank, nranks, cudaDev, &c);
+  if (r != rescclSuccess) return r;
+  std::vector<char> mine(sizeof(Blob)), all(sizeof(Blob) * nranks);
+  size_t len = mine.size();
+  r = rescclCommGetHandle(c, mine.data(), &len);
+  if (r != rescclSuccess) {
+    rescclCommDestroy(c);
+    return r;
+  }
+  if (allgather(mine.data(), all.data(), sizeof(Blob), ctx) != 0) {
+    rescclCommDestroy(c);
+    fail(rescclSystemError, "allgather callback failed");
+  }
+  std::vector<const void*> hs(nranks);
+  std::vector<size_t> ls(nranks, sizeof(Blob));
+  for (int q = 0; q < nranks; ++q) hs[q] = all.data() + q * sizeof(Blob);
+  r = rescclCommConnect(c, hs.data(), ls.data());
+  if (r != rescclSuccess) {
+    rescclCommDestroy(c);
+    return r;
+  }
+  *out = c;
+  API_END
+}
+
+rescclResult_t rescclCommInitAll(rescclComm_t* comms, int ndev, const int* devlist) {
+  API_BEGIN
+  if (!comms || ndev < 1 || ndev > kMaxR) fail(rescclInvalidArgument, "bad arguments");
+  std::vector<int> devs(ndev, 0);
+  if (devlist)
+    for (int i = 0; i < ndev; ++i) devs[i] = devlist[i];
+  bool all_same = true;
+  for (int i = 1; i < ndev; ++i) all_same &= devs[i] == devs[0];
+  bool all_distinct = true;
+  for (int i = 0; i < ndev; ++i)
+    for (int j = i + 1; j < ndev; ++j) all_distinct &= devs[i] != devs[j];
+  if (!all_same && !all_distinct)
+    fail(rescclInvalidUsage, "devlist must be one device repeated (virtual ranks) or distinct devices");
+  std::vector<rescclComm*> cs;
+  if (all_same && ndev > 1) {
+    Group* G = make_group(devs[0], ndev);
+    for (int r = 0; r < ndev; ++r) {
+      auto c = new rescclComm();
+      c->rank = r;
+      c->nranks = ndev;
+      c->dev = devs[0];
+      c->mode = 1;
+      c->group = G;
+      c->connected = true;
+      c->err_host = G->err_host;
+      c->err_dev = G->err_dev;
+      G->comms.push_back(c);
+      G->refs++;
+      cs.push_back(c);
+    }
+  } else {
+    // distinct devices in one process (or a single rank): peer access + direct pointers
+    for (int r = 0; r < ndev; ++r) {
+      auto c = new rescclComm();
+      c->rank = r;
+      c->nranks = ndev;
+      c->dev = devs[r];
+      c->mode = 2;
+      cuda_check(cudaSetDevice(devs[r]), "cudaSetDevice");
+      for (int q = 0; q < ndev; ++q) {
+        if (q == r) continue;
+        cudaError_t e = cudaDeviceEnablePeerAccess(devs[q], 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+          fail(rescclCudaError, std::string("cudaDeviceEnablePeerAccess: ") + cudaGetErrorString(e));
+        cudaGetLastError();
+      }
+      c->arena_bytes = arena_default();
+      cuda_check(cudaMalloc((void**)&c->arena, c->arena_bytes), "cudaMalloc(arena)");
+      cuda_check(cudaMemset(c->arena, 0, c->arena_bytes), "cudaMemset(arena)");
+      alloc_err_word(&c->err_host, &c->err_dev);
+      cs.push_back(c);
+    }
+    for (auto c : cs) {
+      c->peer_arena.resize(ndev);
+      for (int q = 0; q < ndev; ++q) c->peer_arena[q] = cs[q]->arena;
+      c->peer_opened.assign(ndev, false);
+      c->connected = true;
+      c->peers_local = cs;
+      cuda_check(cudaSetDevice(c->dev), "cudaSetDevice");
+      cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
+    }
+  }
+  for (int r = 0; r < ndev; ++r) comms[r] = cs[r];
+  API_END
+}
+
+rescclResult_t rescclCommDestroy(rescclComm_t comm) {
+  API_BEGIN
+  if (!comm) return rescclSuccess;
+  cudaSetDevice(comm->dev);
+  cudaDeviceSynchronize();
+  if (comm->mode == 1) {
+    Group* G = comm->group;
+    if (--G->refs == 0) {
+      for (auto& kv : G->algos) {
+        for (auto& k : kv.second->kernels)
+          if (k.second.mod) driver().ModuleUnload(k.second.mod);
+        kv.second->kernels.clear();
+        if (kv.second->region_alloc) cudaFree(kv.second->region_alloc);
+      }
+      for (auto e : G->events) cudaEventDestroy(e);
+      cudaFreeHost(G->err_host);
+      for (auto c : G->comms)
+        if (c->scratch) cudaFree(c->scratch);
+      delete G;
+    }
+  } else {
+    for (auto& a : comm->algos) {
+      if (a->s.use_count() == 1)
+        for (auto& k : a->s->kernels)
+          if (k.second.mod) driver().ModuleUnload(k.second.mod);
+    }
+    for (int q = 0; q < (int)comm->peer_opened.size(); ++q)
+      if (comm->peer_opened[q]) cudaIpcCloseMemHandle(comm->peer_arena[q]);
+    if (comm->arena) cudaFree(comm->arena);
+    if (comm->err_host) cudaFreeHost(comm->err_host);
+    if (comm->scratch) cudaFree(comm->scratch);
+  }
+  delete comm;
+  API_END
+}
+
+rescclResult_t rescclCommRank(rescclComm_t comm, int* rank) {
+  API_BEGIN
+  if (!comm || !rank) fail(rescclInvalidArgument, "null argument");
+  *rank = comm->rank;
+  API_END
+}
+
+rescclResult_t rescclCommCount(rescclComm_t comm, int* nranks) {
+  API_BEGIN
+  if (!comm || !nranks) fail(rescclInvalidArgument, "null argument");
+  *nranks = comm->nranks;
+  API_END
+}
+
+rescclResult_t rescclCommGetAsyncError(rescclComm_t comm, rescclResult_t* err) {
+  API_BEGIN
+  if (!comm || !err) fail(rescclInvalidArgument, "null argument");
+  volatile int* w = comm->err_host;
+  *err = (w && *w) ? rescclTimeout : rescclSuccess;
+  API_END
+}
+
+rescclResult_t rescclLoadAlgorithm(rescclComm_t comm, const char* irText, rescclAlgo_t* out) {
+  API_BEGIN
+  if (!comm || !irText) fail(rescclInvalidArgument, "null argument");
+  if (!comm->connected) fail(rescclInvalidUsage, "communicator not connected");
+  rescclAlgo* a = load_algo(comm, irText);
+  if (out) *out = a;
+  API_END
+}
+
+rescclResult_t rescclSetActiveAlgorithm(rescclComm_t comm, rescclAlgo_t algo) {
+  API_BEGIN
+  if (!comm || !algo || algo->comm != comm) fail(rescclInvalidArgument, "algorithm does not belong to comm");
+  comm->active[(int)algo->s->ir.coll] = algo;
+  API_END
+}
+
+rescclResult_t rescclGetPlanInfo(rescclAlgo_t algo, char* json, size_t* len) {
+  API_BEGIN
+  if (!algo) fail(rescclInvalidArgument, "algo is NULL");
+  if (algo->s->json.empty()) algo->s->json = info_json(*algo->s);
+  write_out(algo->s->json, json, len);
+  API_END
+}
+
+rescclResult_t rescclAllReduce(const void* sendbuf, void* recvbuf, size_t count, rescclDataType_t dtype,
+                               rescclRedOp_t op, rescclComm_t comm, void* stream) {
+  API_BEGIN
+  collective(comm, (int)Coll::AllReduce, sendbuf, recvbuf, count, dtype, op, stream);
+  API_END
+}
+
+rescclResult_t rescclAllGather(const void* sendbuf, void* recvbuf, size_t sendcount, rescclDataType_t dtype,
+                               rescclComm_t comm, void* stream) {
+  API_BEGIN
+  collective(comm, (int)Coll::AllGather, sendbuf, recvbuf, sendcount, dtype, rescclSum, stream);
+  API_END
+}
+
+rescclResult_t rescclReduceScatter(const void* sendbuf, void* recvbuf, size_t recvcount, rescclDataType_t dtype,
+                                   rescclRedOp_t op, rescclComm_t comm, void* stream) {
+  API_BEGIN
+  collective(comm, (int)Coll::ReduceScatter, sendbuf, recvbuf, recvcount, dtype, op, stream);
+  API_END
+}
+
+// ------------------------------------------------------------------ host-only tools
+rescclResult_t rescclGenerateIr(const char* name, rescclColl_t coll, int nranks, const char* opts, char* text,
+                                size_t* len) {
+  API_BEGIN
+  if (!name) fail(rescclInvalidArgument, "name is NULL");
+  std::map<std::string, long> o;
+  for (auto& kv : parse_kv(opts)) o[kv.first] = to_long(kv.second, kv.first);
+  Ir ir = generate(name, (Coll)coll, nranks, o);
+  write_out(ir.to_text(), text, len);
+  API_END
+}
+
+rescclResult_t rescclPlanIr(const char* irText, const char* opts, char* json, size_t* len) {
+  API_BEGIN
+  Options o;
+  Plan p = plan_from(irText, opts, &o, nullptr);
+  AlgoShared a;
+  a.opt = o;
+  a.plan = p;
+  a.ir = p.ir;
+  a.lay = make_layout(p, o.fifo_depth, o.instances, o.chunk_bytes);
+  write_out(info_json(a), json, len);
+  API_END
+}
+
+rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo, int rank_hi, char* src,
+                               size_t* len) {
+  API_BEGIN
+  Options o;
+  Plan p = plan_from(irText, opts, &o, nullptr);
+  if (rank_lo < 0 || rank_hi > p.ir.nranks || rank_lo >= rank_hi) fail(rescclInvalidArgument, "bad rank range");
+  Layout L = make_layout(p, o.fifo_depth, o.instances, o.chunk_bytes);
+  CodegenOpts co;
+  co.rank_lo = rank_lo;
+  co.rank_hi = rank_hi;
+  co.nwarps = o.nwarps;
+  write_out(codegen(p, L, co), src, len);
+  API_END
+}
+
+rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataType_t dtype, rescclRedOp_t op,
+                               size_t* cubin_bytes) {
+  API_BEGIN
+  Options o;
+  Plan p = plan_from(irText, opts, &o, nullptr);
+  Layout L = make_layout(p, o.fifo_depth, o.instances, o.chunk_bytes);
+  CodegenOpts co;
+  co.rank_lo = 0;
+  co.rank_hi = p.ir.nranks;
+  co.nwarps = o.nwarps;
+  co.gpu_scope = true;
+  auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, true);
+  if (cubin_bytes) *cubin_bytes = cub.size();
+  API_END
+}
+
+rescclResult_t rescclCheckDeadlock(const char* irText, const char* opts, int K, int n_mb, int* ok) {
+  API_BEGIN
+  if (!ok) fail(rescclInvalidArgument, "ok is NULL");
+  Plan p = plan_from(irText, opts, nullptr, nullptr);
+  *ok = deadlock_free(p, K, n_mb) ? 1 : 0;
+  API_END
+}
+
+}  // extern "C"

@@ -1,0 +1,397 @@
+// ResCCL L0 transport device library for sm_100a.
+//
+// Compiled twice: by NVRTC together with the code the kernel generator emits for
+// one schedule (csrc/plan/codegen.cc), and by nvcc in the build self-test.  It
+// must therefore not include any system header.
+//
+// Execution model (§4.5): one generated kernel per
+// schedule; block -> (rank, TB, instance); a TB is two independent warp groups
+// ("lanes", reading R20): warps [0, W/2) run the send-lane primitive list and warps
+// [W/2, W) the recv-lane list.  Each primitive loops over all micro-batches before
+// the next one starts (task-level execution).  For micro-batch j a
+// primitive
+//   1. waits until every local dependency finished micro-batch j (rule (1)):
+//      ld.acquire on a 64-bit monotone counter >= mb_base + j + 1;
+//   2. waits for payload (recv) in its link FIFO slot and/or for FIFO credit (send):
+//      ld.acquire on the slot flag / on the credit counter the receiver writes back;
+//   3. moves 16-byte vectors (or elements on a misaligned tail): send, recv, rrc
+//      (recvReduceCopy), rrs (recvReduceSend), rcs (recvCopySend), rrcs; bf16/fp16
+//      combine in fp32 and round to nearest even on every store (reading R8);
+//   4. publishes: fence, then the slot flag in the receiver's arena, the credit in
+//      the sender's arena and the local completion counter.
+// FIFOs live in the receiver's arena (one per link and instance, depth K, slot =
+// one micro-batch slice); every 64-bit flag/counter is monotone across calls, so
+// no reset kernel is needed.
+#pragma once
+
+#ifndef RESCCL_MAXR
+#define RESCCL_MAXR 32
+#endif
+
+namespace rdev {
+
+typedef unsigned long long u64;
+typedef long long i64;
+typedef unsigned int u32;
+typedef unsigned short u16;
+
+struct KArgs {
+  char* arena[RESCCL_MAXR];           // plan region of every rank's arena (peer-mapped)
+  const char* sendbuf[RESCCL_MAXR];   // per local rank (virtual mode: every rank)
+  char* recvbuf[RESCCL_MAXR];
+  char* scratch[RESCCL_MAXR];
+  u64 mb_base;                        // micro-batches of this plan issued before this call
+  i64 count;                          // AR: count; AG: sendcount; RS: recvcount (elements)
+  i64 C;                              // algorithm-chunk elements
+  i64 M;                              // micro-batch elements
+  i64 Mi;                             // instance-slice elements
+  int n_mb;
+  int block_base;                     // global block id of blockIdx.x == 0
+  int* err;                           // host-mapped error word
+  u64 timeout_ns;
+};
+
+enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16 };
+enum : int { BufSend = 0, BufRecv = 1, BufScratch = 2 };
+enum : int { CollAllGather = 0, CollReduceScatter = 1, CollAllReduce = 2 };
+enum : int { OpSum = 0, OpMax = 1, OpMin = 2 };
+enum : int { kErrTimeout = 7 };
+
+// ----------------------------------------------------------------------------- memory ops
+#if defined(RESCCL_SCOPE_GPU)
+#define RESCCL_SC ".gpu"
+#else
+#define RESCCL_SC ".sys"
+#endif
+
+__device__ __forceinline__ u64 ld_acquire(const u64* p) {
+  u64 v;
+  asm volatile("ld.acquire" RESCCL_SC ".global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed(u64* p, u64 v) {
+  asm volatile("st.relaxed" RESCCL_SC ".global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void fence_release() { asm volatile("fence.acq_rel" RESCCL_SC ";" ::: "memory"); }
+__device__ __forceinline__ u64 globaltimer() {
+  u64 t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void nanosleep_(u32 ns) { asm volatile("nanosleep.u32 %0;" ::"r"(ns)); }
+
+struct V4 {
+  u32 x, y, z, w;
+};
+__device__ __forceinline__ V4 ld_cg(const V4* p) {
+  V4 v;
+  asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void st_v4(V4* p, const V4& v) {
+  asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+__device__ __forceinline__ u32 ld_cg_b32(const void* p) {
+  u32 v;
+  asm volatile("ld.global.cg.b32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ u16 ld_cg_b16(const void* p) {
+  u16 v;
+  asm volatile("ld.global.cg.b16 %0, [%1];" : "=h"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void st_b32(void* p, u32 v) { asm volatile("st.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory"); }
+__device__ __forceinline__ void st_b16(void* p, u16 v) { asm volatile("st.global.b16 [%0], %1;" ::"l"(p), "h"(v) : "memory"); }
+
+// ----------------------------------------------------------------------------- element types
+// Storage types: int32 / f32 as 32-bit words, f16 / bf16 as 16-bit words.
+struct TI32 { enum { kSize = 4, kKind = 0 }; };
+struct TF32 { enum { kSize = 4, kKind = 1 }; };
+struct TF16 { enum { kSize = 2, kKind = 2 }; };
+struct TBF16 { enum { kSize = 2, kKind = 3 }; };
+
+__device__ __forceinline__ float bf_lo(u32 w) { return __uint_as_float(w << 16); }
+__device__ __forceinline__ float bf_hi(u32 w) { return __uint_as_float(w & 0xFFFF0000u); }
+__device__ __forceinline__ u32 pack_bf16x2(float lo, float hi) {
+  u32 r;
+  asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+__device__ __forceinline__ float h_lo(u32 w) {
+  float f;
+  asm("{.reg .b16 l, h; mov.b32 {l, h}, %1; cvt.f32.f16 %0, l;}" : "=f"(f) : "r"(w));
+  return f;
+}
+__device__ __forceinline__ float h_hi(u32 w) {
+  float f;
+  asm("{.reg .b16 l, h; mov.b32 {l, h}, %1; cvt.f32.f16 %0, h;}" : "=f"(f) : "r"(w));
+  return f;
+}
+__device__ __forceinline__ u32 pack_f16x2(float lo, float hi) {
+  u32 r;
+  asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+__device__ __forceinline__ float bf16_to_f(u16 h) { return __uint_as_float(((u32)h) << 16); }
+__device__ __forceinline__ u16 f_to_bf16(float f) {
+  u16 r;
+  asm("cvt.rn.bf16.f32 %0, %1;" : "=h"(r) : "f"(f));
+  return r;
+}
+__device__ __forceinline__ float f16_to_f(u16 h) {
+  float f;
+  asm("cvt.f32.f16 %0, %1;" : "=f"(f) : "h"(h));
+  return f;
+}
+__device__ __forceinline__ u16 f_to_f16(float f) {
+  u16 r;
+  asm("cvt.rn.f16.f32 %0, %1;" : "=h"(r) : "f"(f));
+  return r;
+}
+
+template <int OP>
+__device__ __forceinline__ float fop(float a, float b) {
+  if (OP == OpSum) return __fadd_rn(a, b);
+  if (OP == OpMax) return fmaxf(a, b);
+  return fminf(a, b);
+}
+template <int OP>
+__device__ __forceinline__ u32 iop(u32 a, u32 b) {
+  if (OP == OpSum) return a + b;  // two's-complement wraparound
+  if (OP == OpMax) return (u32)max((int)a, (int)b);
+  return (u32)min((int)a, (int)b);
+}
+
+// combine one 32-bit word: local (+) incoming
+template <class T, int OP>
+__device__ __forceinline__ u32 combine_w(u32 a, u32 b);
+template <> __device__ __forceinline__ u32 combine_w<TI32, OpSum>(u32 a, u32 b) { return iop<OpSum>(a, b); }
+template <> __device__ __forceinline__ u32 combine_w<TI32, OpMax>(u32 a, u32 b) { return iop<OpMax>(a, b); }
+template <> __device__ __forceinline__ u32 combine_w<TI32, OpMin>(u32 a, u32 b) { return iop<OpMin>(a, b); }
+#define RDEV_F32(OPV) \
+  template <> __device__ __forceinline__ u32 combine_w<TF32, OPV>(u32 a, u32 b) { \
+    return __float_as_uint(fop<OPV>(__uint_as_float(a), __uint_as_float(b))); }
+RDEV_F32(OpSum) RDEV_F32(OpMax) RDEV_F32(OpMin)
+#undef RDEV_F32
+#define RDEV_BF(OPV) \
+  template <> __device__ __forceinline__ u32 combine_w<TBF16, OPV>(u32 a, u32 b) { \
+    return pack_bf16x2(fop<OPV>(bf_lo(a), bf_lo(b)), fop<OPV>(bf_hi(a), bf_hi(b))); }
+RDEV_BF(OpSum) RDEV_BF(OpMax) RDEV_BF(OpMin)
+#undef RDEV_BF
+#define RDEV_H(OPV) \
+  template <> __device__ __forceinline__ u32 combine_w<TF16, OPV>(u32 a, u32 b) { \
+    return pack_f16x2(fop<OPV>(h_lo(a), h_lo(b)), fop<OPV>(h_hi(a), h_hi(b))); }
+RDEV_H(OpSum) RDEV_H(OpMax) RDEV_H(OpMin)
+#undef RDEV_H
+
+template <class T, int OP>
+__device__ __forceinline__ V4 combine_v(const V4& a, const V4& b) {
+  V4 r;
+  r.x = combine_w<T, OP>(a.x, b.x);
+  r.y = combine_w<T, OP>(a.y, b.y);
+  r.z = combine_w<T, OP>(a.z, b.z);
+  r.w = combine_w<T, OP>(a.w, b.w);
+  return r;
+}
+
+// scalar (one element) path for misaligned slices and vector tails
+template <class T, int OP>
+__device__ __forceinline__ void elem_move(int F, const char* A, const char* B, char* D1, char* D2, i64 i) {
+  if (T::kSize == 4) {
+    u32 a = 0, b = 0, v;
+    if (A) a = ld_cg_b32(A + 4 * i);
+    if (B) b = ld_cg_b32(B + 4 * i);
+    v = (F & kReduce) ? combine_w<T, OP>(a, b) : ((F & kRecv) ? b : a);
+    if (D1) st_b32(D1 + 4 * i, v);
+    if (D2) st_b32(D2 + 4 * i, v);
+  } else {
+    u16 a = 0, b = 0, v;
+    if (A) a = ld_cg_b16(A + 2 * i);
+    if (B) b = ld_cg_b16(B + 2 * i);
+    if (F & kReduce) {
+      if (T::kKind == 3)
+        v = f_to_bf16(fop<OP>(bf16_to_f(a), bf16_to_f(b)));
+      else
+        v = f_to_f16(fop<OP>(f16_to_f(a), f16_to_f(b)));
+    } else {
+      v = (F & kRecv) ? b : a;
+    }
+    if (D1) st_b16(D1 + 2 * i, v);
+    if (D2) st_b16(D2 + 2 * i, v);
+  }
+}
+
+// Move n elements: A = local source, B = incoming FIFO slot, D1 = local store target,
+// D2 = outgoing FIFO slot.  Null pointers are unused operands (fixed per primitive).
+template <class T, int OP, int F, int U>
+__device__ __forceinline__ void move(i64 n, const char* A, const char* B, char* D1, char* D2, int tid, int nt) {
+  if (n <= 0) return;
+  const unsigned long long al = (unsigned long long)A | (unsigned long long)B | (unsigned long long)D1 |
+                                (unsigned long long)D2;
+  const i64 bytes = n * T::kSize;
+  i64 nv = 0;
+  if ((al & 15) == 0) {
+    nv = bytes >> 4;
+    const V4* a4 = (const V4*)A;
+    const V4* b4 = (const V4*)B;
+    V4* d1 = (V4*)D1;
+    V4* d2 = (V4*)D2;
+    i64 i = tid;
+    // main body: U independent 16-byte vectors in flight per operand per thread
+    for (; i + (i64)(U - 1) * nt < nv; i += (i64)U * nt) {
+      V4 va[U], vb[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (A) va[u] = ld_cg(a4 + i + (i64)u * nt);
+        if (B) vb[u] = ld_cg(b4 + i + (i64)u * nt);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        V4 v = (F & kReduce) ? combine_v<T, OP>(va[u], vb[u]) : ((F & kRecv) ? vb[u] : va[u]);
+        if (D1) st_v4(d1 + i + (i64)u * nt, v);
+        if (D2) st_v4(d2 + i + (i64)u * nt, v);
+      }
+    }
+    for (; i < nv; i += nt) {
+      V4 va, vb;
+      if (A) va = ld_cg(a4 + i);
+      if (B) vb = ld_cg(b4 + i);
+      V4 v = (F & kReduce) ? combine_v<T, OP>(va, vb) : ((F & kRecv) ? vb : va);
+      if (D1) st_v4(d1 + i, v);
+      if (D2) st_v4(d2 + i, v);
+    }
+  }
+  const i64 e0 = (nv << 4) / T::kSize;
+  for (i64 e = e0 + tid; e < n; e += nt) elem_move<T, OP>(F, A, B, D1, D2, e);
+}
+
+// ----------------------------------------------------------------------------- lane
+struct Lane {
+  const KArgs* a;
+  char* self;       // this rank's plan region
+  int rank, inst, bar, nthreads, tid;
+  volatile int* abort_flag;  // shared memory, per lane
+
+  __device__ __forceinline__ void sync() const {
+    asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(nthreads) : "memory");
+  }
+  // leader only: spin until *p >= target; false on timeout (error word set)
+  __device__ bool wait_ge(const u64* p, u64 target) const {
+    if (ld_acquire(p) >= target) return true;
+    u64 t0 = globaltimer();
+    u32 spins = 0;
+    while (ld_acquire(p) < target) {
+      if (++spins > 64) nanosleep_(32);
+      if ((spins & 1023) == 0 && globaltimer() - t0 > a->timeout_ns) {
+        atomicCAS(a->err, 0, kErrTimeout);
+        return false;
+      }
+    }
+    return true;
+  }
+};
+
+__device__ __forceinline__ u64* at(char* base, i64 off) { return (u64*)(base + off); }
+
+template <int COLL>
+__device__ __forceinline__ i64 chunk_len(const KArgs& a, int c) {
+  if (COLL == CollAllReduce) {
+    i64 l = a.count - (i64)c * a.C;
+    return l < 0 ? 0 : (l > a.C ? a.C : l);
+  }
+  return a.count;
+}
+template <int COLL>
+__device__ __forceinline__ i64 chunk_off(int buf, int c, i64 C) {
+  if (COLL == CollAllReduce) return (i64)c * C;
+  if (COLL == CollAllGather) return buf == BufSend ? 0 : (i64)c * C;
+  return buf == BufRecv ? 0 : (i64)c * C;  // reduce-scatter
+}
+__device__ __forceinline__ char* buf_ptr(const KArgs& a, int rank, int buf) {
+  return buf == BufSend ? (char*)a.sendbuf[rank] : (buf == BufRecv ? a.recvbuf[rank] : a.scratch[rank]);
+}
+
+// One primitive of the schedule: constants emitted by the kernel generator as a
+// literal.  Offsets are bytes inside the plan region of the named rank's arena, for
+// instance 0 (instance i adds i * K * SLOT, i * FLAGSTRIDE or i * 128).
+#ifndef RESCCL_MAXDEPS
+#define RESCCL_MAXDEPS 6
+#endif
+struct PrimDesc {
+  int chunk, src_buf, dst_buf, in_peer, out_peer, ndeps;
+  i64 in_data, in_flag, in_cred, in_pos, in_n;
+  i64 out_data, out_flag, out_cred, out_pos, out_n;
+  i64 ctr;
+  i64 deps[RESCCL_MAXDEPS];
+};
+
+// Layout constants shared by every primitive of a plan (emitted by the generator):
+//   RESCCL_K, RESCCL_I, RESCCL_SLOT, RESCCL_FLAGSTRIDE, RESCCL_COLL
+template <class T, int OP, int F>
+__device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
+  const KArgs& a = *L.a;
+  const int c = d.chunk;
+  const i64 len = chunk_len<RESCCL_COLL>(a, c);
+  const char* A = nullptr;
+  char* D1 = nullptr;
+  if ((F & kCopy) || (F & kReduce) || !(F & kRecv))
+    A = buf_ptr(a, L.rank, d.src_buf) + chunk_off<RESCCL_COLL>(d.src_buf, c, a.C) * T::kSize;
+  if ((F & kCopy) || (F & kStore))
+    D1 = buf_ptr(a, L.rank, d.dst_buf) + chunk_off<RESCCL_COLL>(d.dst_buf, c, a.C) * T::kSize;
+  if (F & kCopy) {
+    if (A == D1) return true;  // in-place: own chunk already in place
+    for (int j = 0; j < a.n_mb; ++j) {
+      i64 lo = (i64)j * a.M + (i64)L.inst * a.Mi;
+      i64 hi = lo + a.Mi;
+      if (hi > (i64)(j + 1) * a.M) hi = (i64)(j + 1) * a.M;
+      if (hi > len) hi = len;
+      if (lo > hi) lo = hi;
+      move<T, OP, kCopy, 4>(hi - lo, A + lo * T::kSize, nullptr, D1 + lo * T::kSize, nullptr, L.tid, L.nthreads);
+    }
+    return true;
+  }
+  char* in_data = L.self + d.in_data + (i64)L.inst * RESCCL_K * RESCCL_SLOT;
+  u64* in_flag = at(L.self, d.in_flag + (i64)L.inst * RESCCL_FLAGSTRIDE);
+  u64* in_cred = (F & kRecv) ? at(a.arena[d.in_peer], d.in_cred + (i64)L.inst * 128) : nullptr;
+  char* peer = (F & kSend) ? a.arena[d.out_peer] : nullptr;
+  char* out_data = (F & kSend) ? peer + d.out_data + (i64)L.inst * RESCCL_K * RESCCL_SLOT : nullptr;
+  u64* out_flag = (F & kSend) ? at(peer, d.out_flag + (i64)L.inst * RESCCL_FLAGSTRIDE) : nullptr;
+  u64* out_cred = at(L.self, d.out_cred + (i64)L.inst * 128);
+  u64* ctr = at(L.self, d.ctr + (i64)L.inst * 128);
+  const u64 mb_base = a.mb_base;
+  for (int j = 0; j < a.n_mb; ++j) {
+    const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
+    const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
+    if (L.tid == 0) {
+      bool ok = true;
+      for (int k = 0; k < d.ndeps && ok; ++k)
+        ok = L.wait_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), mb_base + j + 1);
+      if (ok && (F & kRecv)) ok = L.wait_ge(in_flag + (in_seq % RESCCL_K), in_seq + 1);
+      if (ok && (F & kSend) && out_seq + 1 > (u64)RESCCL_K) ok = L.wait_ge(out_cred, out_seq + 1 - RESCCL_K);
+      if (!ok) *L.abort_flag = 1;
+    }
+    L.sync();
+    if (*L.abort_flag) return false;
+    i64 lo = (i64)j * a.M + (i64)L.inst * a.Mi;
+    i64 hi = lo + a.Mi;
+    if (hi > (i64)(j + 1) * a.M) hi = (i64)(j + 1) * a.M;
+    if (hi > len) hi = len;
+    if (lo > hi) lo = hi;
+    const char* Aj = A ? A + lo * T::kSize : nullptr;
+    char* D1j = D1 ? D1 + lo * T::kSize : nullptr;
+    const char* Bj = (F & kRecv) ? in_data + (in_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
+    char* D2j = (F & kSend) ? out_data + (out_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
+    move<T, OP, F, 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
+    L.sync();
+    if (L.tid == 0) {
+      fence_release();
+      if (F & kSend) st_relaxed(out_flag + (out_seq % RESCCL_K), out_seq + 1);
+      if (F & kRecv) st_relaxed(in_cred, in_seq + 1);
+      if (d.ctr >= 0) st_relaxed(ctr, mb_base + j + 1);
+    }
+  }
+  return true;
+}
+
+}  // namespace rdev

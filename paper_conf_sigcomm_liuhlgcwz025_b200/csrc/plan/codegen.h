@@ -1,0 +1,56 @@
+// ResCCL lightweight kernel generation (§4.5).
+//
+// The three-level paradigm "rank -> TB -> pipeline index" is lowered into one
+// CUDA translation unit per schedule: block b -> (rank, TB, instance); each TB's
+// send and recv lanes are straight-line lists of `rdev::run<T, OP, Pk>` calls
+// sorted by pipeline index, every Pk a constexpr descriptor (chunk, buffers, FIFO
+// offsets, link positions, counters, dependency waits).  There is no interpreter:
+// every peer, chunk id, FIFO offset and dependency is a compile-time constant;
+// only buffers, sizes and the micro-batch base are kernel arguments.
+#pragma once
+
+#include <cstdint>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "plan.h"
+
+namespace resccl {
+
+struct Layout {
+  int K = 4;               // FIFO depth (slots per link and instance)
+  int I = 1;               // instances (paper's nChannels / "Instance")
+  int64_t chunk_bytes = 1 << 20;  // Table 2 ChunkSize
+  int64_t slot = 0;        // bytes per FIFO slot
+  int64_t flagstride = 0;  // bytes of flags per (link, instance)
+  // per rank
+  std::vector<std::map<int, int>> send_idx, recv_idx;  // peer -> connection index
+  std::vector<std::vector<int>> ctr_slot;              // prim -> counter slot (-1: none)
+  std::vector<int64_t> cred_base, ctr_base, flag_base, data_base, bytes;
+  int64_t region_bytes = 0;  // max over ranks (regions sit at the same arena offset)
+  // TB geometry
+  std::vector<int> ctas;        // per rank
+  std::vector<int> pair_start;  // per rank: index of (rank, cta 0) among all (rank, cta) pairs
+  int total_pairs = 0;
+};
+
+Layout make_layout(const Plan& p, int K, int I, int64_t chunk_bytes);
+
+struct CodegenOpts {
+  int rank_lo = 0, rank_hi = 0;  // ranks [lo, hi) get code
+  bool gpu_scope = false;        // all ranks on one device (virtual ranks): .gpu-scope flags
+  int nwarps = 16;
+};
+
+// Device code (without the L0 library text, which the runtime prepends).
+std::string codegen(const Plan& p, const Layout& L, const CodegenOpts& o);
+
+// Host geometry of one call (reading R6; identical to the oracle's).
+struct Geometry {
+  int64_t C = 0, M = 0, Mi = 0;
+  int n_mb = 0;
+};
+Geometry geometry(Coll coll, int nranks, int64_t count, int elt, int64_t chunk_bytes, int instances);
+
+}  // namespace resccl

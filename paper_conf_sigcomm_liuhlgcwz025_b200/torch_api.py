@@ -1,0 +1,110 @@
+"""Thin tensor-level helpers over the C ABI (argument marshalling only).
+
+``Communicator`` wraps one rank's ``rescclComm_t``; ``VirtualGroup`` wraps the
+single-process virtual ranks of one GPU (``rescclCommInitAll`` with a repeated
+device).  ``init_process_group_comm`` bootstraps a multi-process communicator by
+exchanging the connection blobs with ``torch.distributed.all_gather_object``.
+"""
+from __future__ import annotations
+
+from typing import List, Optional, Sequence
+
+import paper_conf_sigcomm_liuhlgcwz025_b200 as _r
+
+_TORCH_DT = {"torch.int32": _r.rescclInt32, "torch.float32": _r.rescclFloat32,
+             "torch.float16": _r.rescclFloat16, "torch.bfloat16": _r.rescclBfloat16}
+
+
+def dtype_of(t) -> int:
+    d = _TORCH_DT.get(str(t.dtype))
+    if d is None:
+        raise TypeError(f"unsupported dtype {t.dtype}")
+    return d
+
+
+def _stream(stream) -> int:
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    return stream if isinstance(stream, int) else stream.cuda_stream
+
+
+class Communicator:
+    def __init__(self, handle: int):
+        self.handle = handle
+        self.rank = _r.rescclCommRank(handle)
+        self.nranks = _r.rescclCommCount(handle)
+        self.algos = []
+
+    def load(self, ir_text: str) -> int:
+        a = _r.rescclLoadAlgorithm(self.handle, ir_text)
+        self.algos.append(a)
+        return a
+
+    def allreduce(self, send, recv, op: str = "sum", stream=None):
+        assert send.is_cuda and recv.is_cuda and send.numel() == recv.numel()
+        _r.rescclAllReduce(send.data_ptr(), recv.data_ptr(), send.numel(), dtype_of(send), _r.OPS[op],
+                           self.handle, _stream(stream))
+
+    def allgather(self, send, recv, stream=None):
+        assert recv.numel() == send.numel() * self.nranks
+        _r.rescclAllGather(send.data_ptr(), recv.data_ptr(), send.numel(), dtype_of(send), self.handle,
+                           _stream(stream))
+
+    def reducescatter(self, send, recv, op: str = "sum", stream=None):
+        assert send.numel() == recv.numel() * self.nranks
+        _r.rescclReduceScatter(send.data_ptr(), recv.data_ptr(), recv.numel(), dtype_of(send), _r.OPS[op],
+                               self.handle, _stream(stream))
+
+    def async_error(self) -> int:
+        return _r.rescclCommGetAsyncError(self.handle)
+
+    def destroy(self):
+        if self.handle:
+            _r.rescclCommDestroy(self.handle)
+            self.handle = 0
+
+
+class VirtualGroup:
+    """N virtual ranks on one GPU; every collective is issued for all ranks and runs
+    as one kernel (see resccl.h, "Execution modes")."""
+
+    def __init__(self, nranks: int, device: int = 0):
+        self.comms = [Communicator(h) for h in _r.rescclCommInitAll([device] * nranks)]
+        self.nranks = nranks
+
+    def load(self, ir_text: str) -> List[int]:
+        return [c.load(ir_text) for c in self.comms]
+
+    def plan_info(self) -> dict:
+        return _r.rescclGetPlanInfo(self.comms[0].algos[-1])
+
+    def allreduce(self, sends: Sequence, recvs: Sequence, op: str = "sum", stream=None):
+        for c, s, r in zip(self.comms, sends, recvs):
+            c.allreduce(s, r, op, stream)
+
+    def allgather(self, sends, recvs, stream=None):
+        for c, s, r in zip(self.comms, sends, recvs):
+            c.allgather(s, r, stream)
+
+    def reducescatter(self, sends, recvs, op: str = "sum", stream=None):
+        for c, s, r in zip(self.comms, sends, recvs):
+            c.reducescatter(s, r, op, stream)
+
+    def async_error(self) -> int:
+        return self.comms[0].async_error()
+
+    def destroy(self):
+        for c in self.comms:
+            c.destroy()
+
+
+def init_process_group_comm(rank: int, nranks: int, device: int, group=None) -> Communicator:
+    """Multi-process bootstrap: Create -> GetHandle -> all_gather_object -> Connect."""
+    import torch.distributed as dist
+    h = _r.rescclCommCreate(rank, nranks, device)
+    blob = _r.rescclCommGetHandle(h)
+    blobs: List[Optional[bytes]] = [None] * nranks
+    dist.all_gather_object(blobs, blob, group=group)
+    _r.rescclCommConnect(h, blobs)
+    return Communicator(h)

@@ -1,0 +1,205 @@
+"""GPU parity: the CUDA path (C ABI -> generated sm_100a kernels) vs the CPU oracle.
+
+Bit-exact against the oracle's schedule replay for every dtype (reading R8 makes
+16-bit results exact too), and within the north_star tolerance against the naive
+definition.  Virtual ranks of cuda:0 execute the same generated kernels as the
+multi-GPU path (one launch holds every rank's CTAs)."""
+import numpy as np
+import pytest
+
+import resccl_inputs as inp
+from oracle import definition, ir as oir, lower, numerics, replay
+
+from gpu_helpers import definition_expect, oracle_expect, run_virtual
+
+pytestmark = pytest.mark.gpu
+
+R = None
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    global R
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as mod
+    R = mod
+
+
+def _hdr(g, **kw):
+    for k, v in kw.items():
+        g.extra[k] = str(v)
+    return g.to_text()
+
+
+def _check_bytes(outs, exp, coll, n, count):
+    for r in range(n):
+        a, b = outs[r], exp[r]
+        assert a.shape == b.shape, (r, a.shape, b.shape)
+        if not np.array_equal(a.view(np.uint8), b.view(np.uint8)):
+            bad = np.nonzero(a.view(np.uint8) != b.view(np.uint8))[0]
+            raise AssertionError(f"rank {r}: {bad.size} bytes differ, first at byte {bad[0]}: "
+                                 f"gpu {a[bad[0] // a.itemsize]} oracle {b[bad[0] // b.itemsize]}")
+
+
+def test_config1_ring_allreduce_4096_fp32_2ranks():
+    """BASELINE configs[0]: ring AR of 4096 fp32, 2 ranks, 1 TB, 4 chunks (2 algorithm
+    chunks x 2 micro-batches of 1024 elements, reading R7)."""
+    g = oir.ring_allreduce(2)
+    text = _hdr(g, chunkbytes=4096, instances=1)
+    xs = inp.all_inputs("float32", 0, 2, 4096)
+    outs, info, err = run_virtual(R, text, "allreduce", xs, "float32", 4096)
+    assert err == 0
+    assert info["ctas"] == [1, 1] and info["blocks_per_rank"] == [1, 1]
+    exp = oracle_expect(g, xs, "float32", 4096, chunk_bytes=4096)
+    _check_bytes(outs, exp, "allreduce", 2, 4096)
+    # N = 2: a single commutative add -> also bit-exact to the definition (c5)
+    _check_bytes(outs, definition.allreduce(xs, "float32"), "allreduce", 2, 4096)
+
+
+ALGOS = [
+    ("ring", "allreduce", 2, {}), ("ring", "allreduce", 3, {}), ("ring", "allreduce", 8, {}),
+    ("ring", "allgather", 8, {}), ("ring", "reducescatter", 8, {}),
+    ("dbt", "allreduce", 8, {}), ("hm", "allreduce", 8, {"g": 4}), ("hm", "allgather", 8, {"g": 4}),
+    ("synth", "allgather", 8, {"seed": 0, "fanout": 2}), ("synth", "reducescatter", 8, {"seed": 3, "fanout": 3}),
+]
+
+
+def _inputs(coll, dtype, n, count, seed=1, mode="uniform"):
+    m = count * n if coll == "reducescatter" else count
+    return inp.all_inputs(dtype, seed, n, m, mode)
+
+
+@pytest.mark.parametrize("name,coll,n,kw", ALGOS)
+@pytest.mark.parametrize("dtype", ["float32", "bfloat16"])
+def test_algorithms_bit_exact_vs_replay(name, coll, n, kw, dtype):
+    """Several tiles, several micro-batches and instances, ragged tail."""
+    g = oir.generate(name, coll, n, **kw)
+    count = 3 * 4096 + 77
+    text = _hdr(g, chunkbytes=4096, instances=2, fifodepth=2)
+    xs = _inputs(coll, dtype, n, count)
+    outs, info, err = run_virtual(R, text, coll, xs, dtype, count)
+    assert err == 0
+    exp = oracle_expect(g, xs, dtype, count, chunk_bytes=4096, instances=2, K=2)
+    _check_bytes(outs, exp, coll, n, count)
+
+
+@pytest.mark.parametrize("name,coll,n,kw", ALGOS)
+def test_algorithms_int32_exact_vs_definition(name, coll, n, kw):
+    g = oir.generate(name, coll, n, **kw)
+    count = 10000
+    text = _hdr(g, chunkbytes=8192, instances=3)
+    xs = _inputs(coll, "int32", n, count, mode="wrap")
+    outs, _, err = run_virtual(R, text, coll, xs, "int32", count)
+    assert err == 0
+    _check_bytes(outs, definition_expect(coll, xs, "int32"), coll, n, count)
+
+
+@pytest.mark.parametrize("dtype", ["float16", "float32", "bfloat16", "int32"])
+@pytest.mark.parametrize("op", ["sum", "max", "min"])
+def test_dtypes_and_ops_ring(dtype, op):
+    g = oir.ring_allreduce(4)
+    count = 5000
+    text = _hdr(g, chunkbytes=2048, instances=2)
+    xs = _inputs("allreduce", dtype, 4, count)
+    outs, _, err = run_virtual(R, text, "allreduce", xs, dtype, count, op=op)
+    assert err == 0
+    exp = oracle_expect(g, xs, dtype, count, op=op, chunk_bytes=2048, instances=2)
+    _check_bytes(outs, exp, "allreduce", 4, count)
+
+
+@pytest.mark.parametrize("name,coll,n,kw", ALGOS[2:8])
+@pytest.mark.parametrize("dtype,rtol", [("float32", 1e-5), ("bfloat16", 2e-2)])
+def test_tolerance_vs_naive_definition(name, coll, n, kw, dtype, rtol):
+    """north_star: within 1e-5 (fp32) / 2e-2 (bf16) relative of naive-order summation,
+    with the cancellation-safe bound |g - ref| <= rtol * sum_k |x_k|."""
+    if coll == "allgather":
+        pytest.skip("no arithmetic")
+    g = oir.generate(name, coll, n, **kw)
+    count = 20000
+    xs = _inputs(coll, dtype, n, count, seed=5)
+    outs, _, err = run_virtual(R, _hdr(g, chunkbytes=16384, instances=2), coll, xs, dtype, count)
+    assert err == 0
+    ref = definition_expect(coll, xs, dtype)
+    den = definition.abs_sum(xs, dtype)
+    for r in range(n):
+        d = den if coll == "allreduce" else den[r * count:(r + 1) * count]
+        diff = np.abs(numerics.to_f32(outs[r], dtype).astype(np.float64) -
+                      numerics.to_f32(ref[r], dtype).astype(np.float64))
+        assert np.all(diff <= rtol * d + 1e-30)
+
+
+@pytest.mark.parametrize("coll", ["allreduce", "allgather", "reducescatter"])
+@pytest.mark.parametrize("count", [1, 7, 8, 129, 4097])
+def test_edge_counts_and_inplace(coll, count):
+    """Tails: counts below N, not multiples of the vector width; in-place variants."""
+    n = 8
+    g = oir.generate("ring", coll, n)
+    dtype = "bfloat16"
+    xs = _inputs(coll, dtype, n, count, seed=9)
+    for inplace in (False, True):
+        outs, _, err = run_virtual(R, _hdr(g, chunkbytes=1024, instances=2), coll, xs, dtype, count,
+                                   inplace=inplace)
+        assert err == 0
+        exp = oracle_expect(g, xs, dtype, count, chunk_bytes=1024, instances=2)
+        _check_bytes(outs, exp, coll, n, count)
+
+
+def test_count_zero_is_noop():
+    import torch
+    grp = R.VirtualGroup(4, 0)
+    try:
+        t = [torch.zeros(1, device="cuda:0") for _ in range(4)]
+        for c in grp.comms:
+            R.rescclAllReduce(t[0].data_ptr(), t[0].data_ptr(), 0, R.rescclFloat32, R.rescclSum, c.handle, 0)
+        torch.cuda.synchronize()
+    finally:
+        grp.destroy()
+
+
+def test_repeated_calls_monotone_flags():
+    """Flags/counters are monotone across calls (no reset kernel): 5 back-to-back calls
+    with different sizes reuse the FIFOs correctly."""
+    import torch
+    from gpu_helpers import to_numpy, to_torch
+    n = 4
+    g = oir.ring_allreduce(n)
+    text = _hdr(g, chunkbytes=2048, instances=2, fifodepth=2)
+    grp = R.VirtualGroup(n, 0)
+    try:
+        grp.load(text)
+        for it, count in enumerate([5000, 100, 9999, 4096, 1]):
+            xs = _inputs("allreduce", "float32", n, count, seed=it)
+            s = [to_torch(x, "float32") for x in xs]
+            rv = [torch.empty_like(x) for x in s]
+            grp.allreduce(s, rv)
+            torch.cuda.synchronize()
+            exp = oracle_expect(g, xs, "float32", count, chunk_bytes=2048, instances=2, K=2)
+            _check_bytes([to_numpy(t, "float32") for t in rv], exp, "allreduce", n, count)
+        assert grp.async_error() == 0
+    finally:
+        grp.destroy()
+
+
+@pytest.mark.parametrize("budget", [1, 2, 4, 8, 16])
+def test_tb_budget_sweep_hm_and_dbt(budget):
+    """C3: DBT and HM 2x4 AllReduce under a TB budget; result independent of the plan."""
+    for g in (oir.dbt_allreduce(8), oir.hm_allreduce(2, 4)):
+        count = 40000
+        text = _hdr(g, chunkbytes=8192, tbbudget=budget)
+        xs = _inputs("allreduce", "bfloat16", 8, count, seed=budget)
+        outs, info, err = run_virtual(R, text, "allreduce", xs, "bfloat16", count)
+        assert err == 0
+        assert max(info["blocks_per_rank"]) <= max(budget, max(info["ctas"]))
+        exp = oracle_expect(g, xs, "bfloat16", count, chunk_bytes=8192, instances=info["instances"],
+                            model=info["linkmodel"])
+        _check_bytes(outs, exp, "allreduce", 8, count)
+
+
+def test_load_rejects_bad_ir():
+    grp = R.VirtualGroup(2, 0)
+    try:
+        with pytest.raises(R.ResCCLError):
+            grp.comms[0].load("algo name=x coll=allreduce nranks=3 nchunks=3\n")
+        with pytest.raises(R.ResCCLError):
+            grp.comms[0].load("algo name=x coll=allreduce nranks=2 nchunks=2\nt 0 1 0 0 rrc\nt 1 0 0 0 rrc\n")
+    finally:
+        grp.destroy()
