@@ -1,0 +1,407 @@
+#!/usr/bin/env python
+"""ResCCL bench: AllReduce bus bandwidth of the generated primitive-level kernels.
+
+Contract (see the task's bench.py section):
+  python bench.py --gpus N --steps K --warmup W [--impl resccl|reference]
+prints ONE JSON line on rank 0.
+
+Workload
+  N = 1  (default): BASELINE configs[1]'s ring AllReduce at 8 ranks, run as 8 virtual
+         ranks on cuda:0 (every rank's buffers and FIFOs in one B200's HBM; one
+         generated kernel holds all ranks' CTAs).  bf16, 256 MiB per rank.
+  N > 1  (torchrun, one process per GPU): N real ranks over CUDA-IPC peer memory
+         (NVLink), same algorithm and per-rank size.
+A step = one AllReduce of the whole buffer (every §8(a) row of the hot path runs in
+it: IR -> plan are load-time; the generated kernel's primitives are the step).
+
+busBW = algBW * 2(N-1)/N with algBW = S / t (nccl-tests convention).
+Inputs are larger than L2 (126 MB) on every rank, so no L2 flush is needed.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK_HBM = 6650.0
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="resccl", choices=["resccl", "reference"])
+    p.add_argument("--algo", default="ring", choices=["ring", "dbt", "hm"])
+    p.add_argument("--vranks", type=int, default=8, help="virtual ranks at --gpus 1")
+    p.add_argument("--size-mb", type=float, default=256.0, help="MiB per rank")
+    p.add_argument("--dtype", default="bfloat16", choices=["bfloat16", "float32", "float16", "int32"])
+    p.add_argument("--instances", type=int, default=0, help="0 = auto")
+    p.add_argument("--chunk-bytes", type=int, default=0)
+    p.add_argument("--fifo-depth", type=int, default=0)
+    p.add_argument("--nwarps", type=int, default=0)
+    p.add_argument("--tma", type=int, default=-1, help="-1 = library default (on)")
+    p.add_argument("--e2e-steps", type=int, default=3)
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--sweep", default="", help="comma-separated MiB sizes for an extra busBW sweep")
+    return p.parse_args()
+
+
+def load_peaks():
+    try:
+        with open(PEAKS_FILE) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return FALLBACK_HBM, "fallback"
+
+
+ELT = {"bfloat16": 2, "float16": 2, "float32": 4, "int32": 4}
+
+
+def ir_text(R, algo: str, n: int, opts: dict) -> str:
+    extra = "g=4" if algo == "hm" else ""
+    text = R.rescclGenerateIr(algo, "allreduce", n, extra)
+    hdr, rest = text.split("\n", 1)
+    for k, v in opts.items():
+        if v is not None:
+            hdr += f" {k}={v}"
+    return hdr + "\n" + rest
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q, "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        time.sleep(0.25)
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        time.sleep(0.15)
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------- CPU oracle leg
+
+def cpu_oracle_sample(algo: str, n: int, dtype: str, budget_s: float = 12.0):
+    """Time the oracle (schedule replay, as it stands) on a bounded sample of the same
+    workload; returns (busBW-equivalent GB/s, seconds per call, sample description)."""
+    import resccl_inputs as inp
+    from oracle import ir as oir, lower, replay
+    g = oir.generate(algo, "allreduce", n, **({"g": 4} if algo == "hm" else {}))
+    pl = lower.lower(g)
+    count = (4 << 20) // ELT[dtype]          # 4 MiB per rank
+    xs = inp.all_inputs(dtype, 0, n, count)
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        replay.replay(pl, xs, dtype, count, chunk_bytes=1 << 20, instances=1, K=4)
+        reps += 1
+        if time.perf_counter() - t0 > budget_s:
+            break
+    dt = (time.perf_counter() - t0) / reps
+    S = count * ELT[dtype]
+    bus = S / dt * 2 * (n - 1) / n / 1e9
+    return bus, dt, f"{algo} allreduce, {n} ranks x {S >> 20} MiB {dtype}, {reps} replay(s), 1 thread"
+
+
+def reference_impl(args):
+    """--impl reference: the oracle timed on the host cores (tier framing)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    n = args.vranks if args.gpus == 1 else args.gpus
+    vals = []
+    for _ in range(args.warmup):
+        cpu_oracle_sample(args.algo, n, args.dtype, budget_s=0.0)
+    t_all = []
+    for _ in range(args.steps):
+        bus, dt, desc = cpu_oracle_sample(args.algo, n, args.dtype, budget_s=0.0)
+        vals.append(bus)
+        t_all.append(dt)
+    value = statistics.mean(vals)
+    line = {
+        "impl": "reference", "metric": "allreduce busBW", "value": round(value, 4), "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(1e3 * statistics.mean(t_all), 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": {"bfloat16": "bf16"}.get(args.dtype, args.dtype),
+        "data": "synthetic",
+        "config": {"workload": f"{args.algo} allreduce, {n} ranks, CPU oracle schedule replay "
+                               f"(bounded sample: 4 MiB per rank)", "nranks": n},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": desc},
+        "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------- ResCCL leg
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return reference_impl(args)
+    import torch
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    multi = world > 1
+    if multi:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("gloo")
+    dev = torch.device("cuda", local if multi else 0)
+    n = world if multi else args.vranks
+    elt = ELT[args.dtype]
+    count = int(args.size_mb * (1 << 20)) // elt
+    S = count * elt
+    tdt = getattr(torch, args.dtype)
+    # default tuning: fill the SMs at N=1 (8 virtual ranks share one GPU)
+    # default tuning (r01 sweep, profiles/r01_*): 16 instances x 8 virtual ranks = 128 CTAs,
+    # 2 MiB transfer chunks, FIFO depth 2 (keeps the FIFOs L2-resident)
+    inst = args.instances or 16
+    opts = {"instances": inst, "chunkbytes": args.chunk_bytes or (2 << 20), "fifodepth": args.fifo_depth or 2,
+            "nwarps": args.nwarps or None, "tma": None if args.tma < 0 else args.tma}
+    text = ir_text(R, args.algo, n, opts)
+
+    if multi:
+        comm = R.init_process_group_comm(rank, world, local)
+        algo = comm.load(text)
+        comms = [comm]
+    else:
+        grp = R.VirtualGroup(n, 0)
+        grp.load(text)
+        comms = grp.comms
+        algo = comms[0].algos[-1]
+    info = R.rescclGetPlanInfo(algo)
+    blocks = info["blocks_per_rank"]
+
+    gen = torch.Generator(device=dev)
+    gen.manual_seed(1234 + rank)
+    my_ranks = [rank] if multi else list(range(n))
+    sends = {r: (torch.rand(count, generator=gen, device=dev, dtype=torch.float32) * 2 - 1).to(tdt)
+             if tdt.is_floating_point else torch.randint(-2 ** 20, 2 ** 20, (count,), device=dev, dtype=tdt)
+             for r in my_ranks}
+    recvs = {r: torch.empty_like(sends[r]) for r in my_ranks}
+    stream = torch.cuda.current_stream(dev)
+    sid = stream.cuda_stream
+
+    def step():
+        for r in my_ranks:
+            c = comms[0] if multi else comms[r]
+            c.allreduce(sends[r], recvs[r], stream=sid)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize(dev)
+
+    def barrier():
+        if multi:
+            torch.distributed.barrier()
+
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize(dev)
+    with ClockSampler(dev.index) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            step()
+        ev1.record(stream)
+        torch.cuda.synchronize(dev)
+    barrier()
+    ms = ev0.elapsed_time(ev1) / args.steps
+    if multi:
+        t = torch.tensor([ms], dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+    err = comms[0].async_error()
+    algbw = S / (ms * 1e-3) / 1e9
+    busbw = algbw * 2 * (n - 1) / n
+
+    # ---- end to end: host (pinned) buffers, H2D + collective + D2H inside the timed region
+    e2e = None
+    if args.e2e_steps > 0:
+        hin = {r: sends[r].cpu().pin_memory() for r in my_ranks}
+        hout = {r: torch.empty_like(hin[r]).pin_memory() for r in my_ranks}
+        for _ in range(2):
+            for r in my_ranks:
+                sends[r].copy_(hin[r], non_blocking=True)
+            step()
+            for r in my_ranks:
+                hout[r].copy_(recvs[r], non_blocking=True)
+        torch.cuda.synchronize(dev)
+        barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            for r in my_ranks:
+                sends[r].copy_(hin[r], non_blocking=True)
+            step()
+            for r in my_ranks:
+                hout[r].copy_(recvs[r], non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        ems = e0.elapsed_time(e1) / args.e2e_steps
+        if multi:
+            t = torch.tensor([ems], dtype=torch.float64)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e_bus = S / (ems * 1e-3) / 1e9 * 2 * (n - 1) / n
+        e2e = {"value": round(e2e_bus, 3), "unit": "GB/s", "h2d_bytes_per_step": S * len(my_ranks),
+               "d2h_bytes_per_step": S * len(my_ranks), "ms_per_step": round(ems, 3)}
+
+    # ---- extra size sweep (busBW vs size)
+    sweep = {}
+    if args.sweep:
+        for mb in [float(x) for x in args.sweep.split(",") if x]:
+            cnt = int(mb * (1 << 20)) // elt
+            s2 = {r: sends[r][:cnt] for r in my_ranks}
+            r2 = {r: recvs[r][:cnt] for r in my_ranks}
+            for _ in range(3):
+                for r in my_ranks:
+                    (comms[0] if multi else comms[r]).allreduce(s2[r], r2[r], stream=sid)
+            torch.cuda.synchronize(dev)
+            barrier()
+            a0 = torch.cuda.Event(enable_timing=True)
+            a1 = torch.cuda.Event(enable_timing=True)
+            reps = 10
+            a0.record(stream)
+            for _ in range(reps):
+                for r in my_ranks:
+                    (comms[0] if multi else comms[r]).allreduce(s2[r], r2[r], stream=sid)
+            a1.record(stream)
+            torch.cuda.synchronize(dev)
+            t_ms = a0.elapsed_time(a1) / reps
+            sweep[f"{mb:g}MiB"] = round(cnt * elt / (t_ms * 1e-3) / 1e9 * 2 * (n - 1) / n, 2)
+
+    if rank != 0:
+        if multi:
+            torch.distributed.destroy_process_group()
+        return
+
+    # ---- roofline (dominant and only kernel: the generated schedule kernel)
+    peak, peak_src = load_peaks()
+    nr = n
+    if multi:
+        # per GPU: NVLink egress 2(N-1)/N S is the bound (900 GB/s/dir nominal)
+        algo_bytes = 2 * (nr - 1) / nr * S
+        roof = {"bound": "nvlink", "achieved": round(algo_bytes / (ms * 1e-3) / 1e9, 2), "peak": 900.0,
+                "unit": "GB/s", "frac": round(algo_bytes / (ms * 1e-3) / 1e9 / 900.0, 4), "traffic": None,
+                "peak_source": "nominal NVLink 5 per direction (measured ref 770 GB/s)"}
+    else:
+        # HBM bytes the staged task-level ring AR must move per rank:
+        # the user-buffer traffic of its primitives -- RS hop: send reads s, rrc reads s and
+        # writes s; AG hop: send reads s, recv writes s => 5(N-1)/N * S (s = S/N).  The FIFO
+        # slots (K x slot per link, a few MiB in total) are L2-resident by design and are
+        # reported separately as l2_fifo_bytes (SURVEY §8(d) d3 counts them: 9(N-1)/N * S).
+        per_rank = 5.0 * (nr - 1) / nr * S
+        algo_bytes = per_rank * nr
+        ach = algo_bytes / (ms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(ach / peak, 4), "traffic": None,
+                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}, burst)",
+                "algorithmic_bytes_per_launch": int(algo_bytes),
+                "l2_fifo_bytes_per_launch": int(4.0 * (nr - 1) / nr * S * nr)}
+    tr = os.environ.get("RESCCL_BENCH_TRAFFIC")
+    if tr:
+        roof["traffic"] = float(tr)
+
+    cpu = None
+    if not args.no_cpu_baseline and not multi:
+        bus_cpu, dt_cpu, desc = cpu_oracle_sample(args.algo, n, args.dtype)
+        cpu = {"value": round(bus_cpu, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc,
+               "s_per_call": round(dt_cpu, 3)}
+
+    sms = sum(blocks) if not multi else blocks[rank]
+    line = {
+        "metric": "allreduce busBW", "value": round(busbw, 2), "unit": "GB/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None,
+        "dtype": {"bfloat16": "bf16", "float16": "f16", "float32": "f32", "int32": "i32"}[args.dtype],
+        "data": "synthetic",
+        "config": {
+            "workload": (f"{args.algo} allreduce, {n} virtual ranks on 1 B200 (all ranks' buffers and FIFOs "
+                         f"in one HBM), {S >> 20} MiB per rank" if not multi else
+                         f"{args.algo} allreduce, {n} GPUs (CUDA-IPC NVLink), {S >> 20} MiB per rank"),
+            "nranks": n, "bytes_per_rank": S, "algo": args.algo, "instances": info["instances"],
+            "chunkbytes": info["chunkbytes"], "fifodepth": info["fifodepth"], "nwarps": info["nwarps"],
+            "linkmodel": info["linkmodel"], "ctas_per_rank": info["ctas"], "blocks_total": sum(blocks),
+            "sms_used": sms, "algbw_gbs": round(algbw, 2), "l2": "inputs > L2 on every rank (no flush)",
+            "parallelism": "virtual-ranks" if not multi else f"ranks{n}",
+        },
+        "roofline": roof,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": args.steps * (1 if not multi else 1),
+        "clocks": clk.summary(),
+        "async_error": err,
+    }
+    if sweep:
+        line["sweep_busbw_gbs"] = sweep
+    print(json.dumps(line), flush=True)
+    if multi:
+        torch.distributed.destroy_process_group()
+    else:
+        grp.destroy()
+
+
+if __name__ == "__main__":
+    main()

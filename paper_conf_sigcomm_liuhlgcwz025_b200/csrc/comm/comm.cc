@@ -74,6 +74,7 @@ struct Driver {
   CUresult (*LaunchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
                            CUstream, void**, void**) = nullptr;
   CUresult (*GetErrorString)(CUresult, const char**) = nullptr;
+  CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
   bool ok = false;
 };
 
@@ -97,6 +98,7 @@ Driver& driver() {
       entry("cuLaunchCooperativeKernel", &d.LaunchCooperativeKernel);
       entry("cuLaunchKernel", &d.LaunchKernel);
       entry("cuGetErrorString", &d.GetErrorString);
+      entry("cuFuncSetAttribute", &d.FuncSetAttribute);
       d.ok = true;
     } catch (Error&) {
       d.ok = false;
@@ -123,6 +125,9 @@ struct Options {
   LinkModel model = LinkModel::Pair;
   bool fuse = true;
   int tb_budget = 0;
+  int tma = 1;
+  int tma_tile = 16384;
+  int tma_stages = 4;
 };
 
 std::map<std::string, std::string> parse_kv(const char* s) {
@@ -156,6 +161,9 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "nwarps") o.nwarps = (int)to_long(v, k);
   else if (k == "fuse") o.fuse = to_long(v, k) != 0;
   else if (k == "tbbudget") o.tb_budget = (int)to_long(v, k);
+  else if (k == "tma") o.tma = (int)to_long(v, k);
+  else if (k == "tmatile") o.tma_tile = (int)to_long(v, k);
+  else if (k == "tmastages") o.tma_stages = (int)to_long(v, k);
   else if (k == "linkmodel") {
     if (v == "pair") o.model = LinkModel::Pair;
     else if (v == "port") o.model = LinkModel::Port;
@@ -170,7 +178,8 @@ Options make_options(const Ir& ir, const char* extra) {
   static const std::pair<const char*, const char*> envs[] = {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
-      {"RESCCL_TB_BUDGET", "tbbudget"}};
+      {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
+      {"RESCCL_TMA_STAGES", "tmastages"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -178,6 +187,9 @@ Options make_options(const Ir& ir, const char* extra) {
   if (o.fifo_depth < 1 || o.fifo_depth > 64) fail(rescclInvalidArgument, "fifodepth must be 1..64");
   if (o.chunk_bytes < 256 || o.chunk_bytes > (1ll << 30)) fail(rescclInvalidArgument, "chunkbytes out of range");
   if (o.nwarps < 2 || o.nwarps > 32 || o.nwarps % 2) fail(rescclInvalidArgument, "nwarps must be even, 2..32");
+  if (o.tma_tile < 1024 || o.tma_tile % 128 || o.tma_stages < 1 || o.tma_stages > 8 ||
+      2 * o.tma_tile * o.tma_stages > 200 * 1024)
+    fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 2*tile*stages <= 200 KiB");
   return o;
 }
 
@@ -263,6 +275,7 @@ std::vector<char> nvrtc_compile(const std::string& gen_src, rescclDataType_t dt,
 struct Kern {
   CUmodule mod = nullptr;
   CUfunction fn = nullptr;
+  int smem = 0;
 };
 
 struct AlgoShared {
@@ -373,7 +386,8 @@ std::string info_json(const AlgoShared& a) {
   std::ostringstream o;
   std::string pj = plan_json(a.plan);
   o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
-    << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"linkmodel\":\""
+    << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"tma\":" << a.opt.tma
+    << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"linkmodel\":\""
     << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
     << ",\"ctas\":[";
   for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];
@@ -393,11 +407,24 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.rank_hi = hi;
   co.gpu_scope = gpu_scope;
   co.nwarps = a.opt.nwarps;
+  co.tma = a.opt.tma;
+  co.tma_tile = a.opt.tma_tile;
+  co.tma_stages = a.opt.tma_stages;
   std::string src = codegen(a.plan, a.lay, co);
+  if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
+    if (FILE* f = fopen((std::string(dump) + "_" + a.ir.name + "_" + coll_name(a.ir.coll) + ".cu").c_str(), "w")) {
+      fputs(src.c_str(), f);
+      fclose(f);
+    }
+  }
   std::vector<char> cubin = nvrtc_compile(src, dt, op, gpu_scope);
   Kern k;
   cu_check(driver().ModuleLoadData(&k.mod, cubin.data()), "cuModuleLoadData");
   cu_check(driver().ModuleGetFunction(&k.fn, k.mod, "resccl_kernel"), "cuModuleGetFunction");
+  k.smem = codegen_smem_bytes(co);
+  if (k.smem > 0)
+    cu_check(driver().FuncSetAttribute(k.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, k.smem),
+             "cuFuncSetAttribute");
   return a.kernels[key] = k;
 }
 
@@ -473,7 +500,7 @@ void ensure_scratch(rescclComm* comm, size_t bytes) {
 
 void launch(Kern& k, int grid, int block, KArgs& args, cudaStream_t s) {
   void* params[] = {&args};
-  cu_check(driver().LaunchCooperativeKernel(k.fn, grid, 1, 1, block, 1, 1, 0, (CUstream)s, params),
+  cu_check(driver().LaunchCooperativeKernel(k.fn, grid, 1, 1, block, 1, 1, k.smem, (CUstream)s, params),
            "cuLaunchCooperativeKernel");
 }
 
@@ -1001,6 +1028,9 @@ rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo
   co.rank_lo = rank_lo;
   co.rank_hi = rank_hi;
   co.nwarps = o.nwarps;
+  co.tma = o.tma;
+  co.tma_tile = o.tma_tile;
+  co.tma_stages = o.tma_stages;
   write_out(codegen(p, L, co), src, len);
   API_END
 }
@@ -1015,6 +1045,9 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
   co.rank_lo = 0;
   co.rank_hi = p.ir.nranks;
   co.nwarps = o.nwarps;
+  co.tma = o.tma;
+  co.tma_tile = o.tma_tile;
+  co.tma_stages = o.tma_stages;
   co.gpu_scope = true;
   auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, true);
   if (cubin_bytes) *cubin_bytes = cub.size();

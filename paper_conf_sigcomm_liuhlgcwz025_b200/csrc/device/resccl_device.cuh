@@ -27,6 +27,9 @@
 #ifndef RESCCL_MAXR
 #define RESCCL_MAXR 32
 #endif
+#ifndef RESCCL_TMA
+#define RESCCL_TMA 1
+#endif
 
 namespace rdev {
 
@@ -103,6 +106,46 @@ __device__ __forceinline__ u16 ld_cg_b16(const void* p) {
 }
 __device__ __forceinline__ void st_b32(void* p, u32 v) { asm volatile("st.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory"); }
 __device__ __forceinline__ void st_b16(void* p, u16 v) { asm volatile("st.global.b16 [%0], %1;" ::"l"(p), "h"(v) : "memory"); }
+
+// ----------------------------------------------------------------------------- TMA bulk copies
+// cp.async.bulk global -> shared (mbarrier complete_tx) and shared -> global (bulk
+// groups).  Used for the pure data-movement primitives (send, recv, rcs, rs, copy):
+// one elected thread per lane keeps up to RESCCL_TMA_STAGES tiles in flight, so the
+// bytes in flight per SM no longer depend on the thread count.
+#ifndef RESCCL_TMA_TILE
+#define RESCCL_TMA_TILE 16384
+#endif
+#ifndef RESCCL_TMA_STAGES
+#define RESCCL_TMA_STAGES 4
+#endif
+__device__ __forceinline__ u32 smem_u32(const void* p) {
+  return (u32)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(u32 bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(u32 bar, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u32 bar, u32 parity) {
+  asm volatile(
+      "{\n.reg .pred p;\nWAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n}\n" ::"r"(bar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_load(u32 dst_smem, const void* src, u32 bytes, u32 bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(dst_smem), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void tma_store(void* dst, u32 src_smem, u32 bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src_smem), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void tma_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void tma_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void tma_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
 
 // ----------------------------------------------------------------------------- element types
 // Storage types: int32 / f32 as 32-bit words, f16 / bf16 as 16-bit words.
@@ -272,6 +315,9 @@ struct Lane {
   char* self;       // this rank's plan region
   int rank, inst, bar, nthreads, tid;
   volatile int* abort_flag;  // shared memory, per lane
+  char* stage;               // this lane's TMA staging buffer (RESCCL_TMA_STAGES tiles)
+  u32 mbar;                  // shared address of this lane's RESCCL_TMA_STAGES mbarriers
+  u32 tma_seq;               // tiles loaded so far (leader only): stage = seq % S, parity = (seq / S) & 1
 
   __device__ __forceinline__ void sync() const {
     asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(nthreads) : "memory");
@@ -310,6 +356,41 @@ __device__ __forceinline__ i64 chunk_off(int buf, int c, i64 C) {
 }
 __device__ __forceinline__ char* buf_ptr(const KArgs& a, int rank, int buf) {
   return buf == BufSend ? (char*)a.sendbuf[rank] : (buf == BufRecv ? a.recvbuf[rank] : a.scratch[rank]);
+}
+
+// Leader-only: copy `bytes` (multiple of 16; 16-byte aligned pointers) from S to D1
+// and/or D2 through the lane's shared-memory stages.
+__device__ __noinline__ void tma_copy(Lane& L, const char* S, char* D1, char* D2, i64 bytes) {
+  const int NS = RESCCL_TMA_STAGES;
+  const i64 TB = RESCCL_TMA_TILE;
+  const i64 ntiles = (bytes + TB - 1) / TB;
+  const u32 sbase = smem_u32(L.stage);
+  const u32 base = L.tma_seq;
+  auto issue = [&](i64 t) {
+    const u32 k = base + (u32)t;
+    const u32 st = k % NS;
+    const i64 off = t * TB;
+    const u32 nb = (u32)((bytes - off) < TB ? (bytes - off) : TB);
+    mbar_expect_tx(L.mbar + 8 * st, nb);
+    tma_load(sbase + st * (u32)TB, S + off, nb, L.mbar + 8 * st);
+  };
+  for (i64 t = 0; t < ntiles && t < NS; ++t) issue(t);
+  for (i64 t = 0; t < ntiles; ++t) {
+    const u32 k = base + (u32)t;
+    const u32 st = k % NS;
+    const i64 off = t * TB;
+    const u32 nb = (u32)((bytes - off) < TB ? (bytes - off) : TB);
+    mbar_wait(L.mbar + 8 * st, (k / NS) & 1);
+    if (D1) tma_store(D1 + off, sbase + st * (u32)TB, nb);
+    if (D2) tma_store(D2 + off, sbase + st * (u32)TB, nb);
+    tma_commit();
+    if (t + NS < ntiles) {
+      tma_wait_read0();
+      issue(t + NS);
+    }
+  }
+  tma_wait_all();
+  L.tma_seq = base + (u32)ntiles;
 }
 
 // One primitive of the schedule: constants emitted by the kernel generator as a
@@ -382,7 +463,23 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
     char* D1j = D1 ? D1 + lo * T::kSize : nullptr;
     const char* Bj = (F & kRecv) ? in_data + (in_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
     char* D2j = (F & kSend) ? out_data + (out_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
-    move<T, OP, F, 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
+#if RESCCL_TMA
+    if (!(F & kReduce)) {
+      // pure data movement: bulk copy the 16-byte-aligned body, threads do the tail
+      const char* Sj = (F & kRecv) ? Bj : Aj;
+      const unsigned long long al = (unsigned long long)Sj | (unsigned long long)D1j | (unsigned long long)D2j;
+      const i64 nb = (al & 15) ? 0 : (((hi - lo) * T::kSize) & ~(i64)15);
+      if (L.tid == 0 && nb > 0) {
+        fence_proxy_async();
+        tma_copy(L, Sj, D1j, D2j, nb);
+        fence_proxy_async();
+      }
+      const i64 e0 = nb / T::kSize;
+      move<T, OP, F, 4>(hi - lo - e0, Aj ? Aj + nb : nullptr, Bj ? Bj + nb : nullptr, D1j ? D1j + nb : nullptr,
+                        D2j ? D2j + nb : nullptr, L.tid, L.nthreads);
+    } else
+#endif
+      move<T, OP, F, 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
     L.sync();
     if (L.tid == 0) {
       fence_release();
