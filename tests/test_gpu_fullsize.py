@@ -1,0 +1,70 @@
+"""Parity at BASELINE's full sizes in bench.py's launch configuration, on sampled
+outputs: every rank's result at sampled positions (random + chunk / micro-batch /
+instance-slice boundaries) equals the oracle's step-order dataflow evaluation of the
+same IR (same association order, R8) on the same seeded inputs."""
+import numpy as np
+import pytest
+
+import resccl_inputs as inp
+from oracle import ir as oir, replay
+
+pytestmark = pytest.mark.gpu
+
+
+def _positions(geo, c, rng, n_rand=3000):
+    L = geo.chunk_len[c]
+    if L == 0:
+        return np.zeros(0, dtype=np.int64)
+    pts = set(rng.integers(0, L, n_rand).tolist())
+    for j in range(geo.n_mb):
+        for i in range(geo.instances):
+            lo, hi = geo.slice(c, j, i)
+            for p in (lo, lo + 1, hi - 2, hi - 1):
+                if 0 <= p < L:
+                    pts.add(p)
+    pts.update([0, L - 1])
+    return np.array(sorted(pts), dtype=np.int64)
+
+
+@pytest.mark.timeout(600)
+@pytest.mark.parametrize("algo,n,size_mb,dtype,opts", [
+    ("ring", 8, 256, "bfloat16", dict(instances=16, chunkbytes=2 << 20, fifodepth=2)),   # bench.py default
+    ("ring", 8, 64, "float32", dict(instances=16, chunkbytes=2 << 20, fifodepth=2)),
+    ("hm", 8, 64, "bfloat16", dict(instances=4, chunkbytes=1 << 20, fifodepth=2)),
+    ("dbt", 8, 64, "float16", dict(instances=4, chunkbytes=1 << 20, fifodepth=2)),
+])
+def test_fullsize_sampled(algo, n, size_mb, dtype, opts):
+    import torch
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    elt = {"bfloat16": 2, "float16": 2, "float32": 4}[dtype]
+    count = size_mb * (1 << 20) // elt
+    g = oir.generate(algo, "allreduce", n, **({"g": 4} if algo == "hm" else {}))
+    for k, v in opts.items():
+        g.extra[k] = str(v)
+    grp = R.VirtualGroup(n, 0)
+    try:
+        grp.load(g.to_text())
+        sends = [inp.rank_input_torch(dtype, 11, r, count) for r in range(n)]
+        recvs = [torch.empty_like(s) for s in sends]
+        for _ in range(2):
+            for t in recvs:
+                t.fill_(float("nan"))
+            grp.allreduce(sends, recvs)
+            torch.cuda.synchronize()
+        assert grp.async_error() == 0
+        geo = replay.Geometry("allreduce", n, count, elt, opts["chunkbytes"], opts["instances"])
+        rng = np.random.default_rng(0)
+        pos = [_positions(geo, c, rng) for c in range(n)]
+        chunk_in = [[inp.rank_input_at(dtype, 11, r, c * geo.C + pos[c]) for c in range(n)] for r in range(n)]
+        exp = replay.dataflow_values(g, chunk_in, dtype)
+        for r in range(n):
+            out = recvs[r]
+            for c in range(n):
+                if pos[c].size == 0:
+                    continue
+                idx = torch.from_numpy(c * geo.C + pos[c]).to(out.device)
+                got = out[idx].cpu()
+                got = got.view(torch.int16).numpy().view(np.uint16) if dtype == "bfloat16" else got.numpy()
+                assert np.array_equal(got.view(np.uint8), exp[r][c].view(np.uint8)), (r, c)
+    finally:
+        grp.destroy()

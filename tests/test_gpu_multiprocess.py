@@ -1,0 +1,94 @@
+"""Multi-process path (one process per rank, CUDA-IPC-mapped peer arenas, .sys-scope
+flags) exercised with every process on cuda:0 -- the gpurun boxes have one GPU; CUDA
+IPC works between processes of one device.  Results are compared with the oracle."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, algo, coll, count, dtype, q):
+    try:
+        import sys
+        root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+        sys.path.insert(0, root)
+        sys.path.insert(0, os.path.join(root, "tests"))
+        import torch
+        import torch.distributed as dist
+        import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+        import resccl_inputs as inp
+        from gpu_helpers import to_numpy, to_torch, poison
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        comm = R.init_process_group_comm(rank, world, 0)
+        text = R.rescclGenerateIr(algo, coll, world)
+        hdr, rest = text.split("\n", 1)
+        comm.load(hdr + " chunkbytes=4096 instances=2 fifodepth=2\n" + rest)
+        m = count * world if coll == "reducescatter" else count
+        x = inp.rank_input(dtype, 3, rank, m)
+        s = to_torch(x, dtype)
+        outs = []
+        for it in range(2):  # two calls: monotone flags across calls
+            n_out = count * world if coll == "allgather" else count
+            r = torch.empty(n_out, dtype=s.dtype, device="cuda:0")
+            poison(r)
+            getattr(comm, coll)(s, r)
+            torch.cuda.synchronize()
+            outs.append(to_numpy(r, dtype))
+        err = comm.async_error()
+        dist.barrier()
+        comm.destroy()
+        dist.destroy_process_group()
+        q.put((rank, outs, err, None))
+    except Exception as e:  # pragma: no cover
+        import traceback
+        q.put((rank, None, None, traceback.format_exc()))
+
+
+@pytest.mark.timeout(240)
+@pytest.mark.parametrize("algo,coll,world", [("ring", "allreduce", 2), ("ring", "allgather", 2),
+                                             ("ring", "reducescatter", 2), ("dbt", "allreduce", 4)])
+def test_ipc_processes_match_oracle(algo, coll, world):
+    import torch.multiprocessing as mp
+    import resccl_inputs as inp
+    from oracle import ir as oir, lower, replay
+    count, dtype = 9000, "float32"
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    env_old = os.environ.get("RESCCL_TIMEOUT_MS")
+    os.environ["RESCCL_TIMEOUT_MS"] = "60000"
+    procs = [ctx.Process(target=_worker, args=(r, world, port, algo, coll, count, dtype, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        rank, outs, err, tb = q.get(timeout=220)
+        assert tb is None, tb
+        res[rank] = (outs, err)
+    for p in procs:
+        p.join(30)
+    if env_old is None:
+        os.environ.pop("RESCCL_TIMEOUT_MS", None)
+    g = oir.generate(algo, coll, world)
+    m = count * world if coll == "reducescatter" else count
+    xs = [inp.rank_input(dtype, 3, r, m) for r in range(world)]
+    exp = replay.replay(lower.lower(g), xs, dtype, count, chunk_bytes=4096, instances=2, K=2)
+    for r in range(world):
+        outs, err = res[r]
+        assert err == 0
+        for o in outs:
+            assert np.array_equal(o.view(np.uint8), exp[r].view(np.uint8)), f"rank {r}"
