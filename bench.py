@@ -347,19 +347,20 @@ def main():
                 "unit": "GB/s", "frac": round(algo_bytes / (ms * 1e-3) / 1e9 / 900.0, 4), "traffic": None,
                 "peak_source": "nominal NVLink 5 per direction (measured ref 770 GB/s)"}
     else:
-        # HBM bytes the staged task-level ring AR must move per rank:
-        # the user-buffer traffic of its primitives -- RS hop: send reads s, rrc reads s and
-        # writes s; AG hop: send reads s, recv writes s => 5(N-1)/N * S (s = S/N).  The FIFO
-        # slots (K x slot per link, a few MiB in total) are L2-resident by design and are
-        # reported separately as l2_fifo_bytes (SURVEY §8(d) d3 counts them: 9(N-1)/N * S).
-        per_rank = 5.0 * (nr - 1) / nr * S
+        # Bytes the staged task-level ring AR moves through the memory system per rank
+        # (DESIGN.md §5.5): RS hop = send (read s, write FIFO s) + rrc
+        # (read FIFO s, read s, write s) = 5s; AG hop = send 2s + recv 2s = 4s; s = S/N
+        # => 9(N-1)/N * S.  Every byte crosses the L2 slices (LTS), whose throughput cap is
+        # what also bounds the measured HBM copy peak, so that peak is the denominator.
+        # dram_algorithmic = the user-buffer share 5(N-1)/N * S (FIFO slots stay in L2).
+        per_rank = 9.0 * (nr - 1) / nr * S
         algo_bytes = per_rank * nr
         ach = algo_bytes / (ms * 1e-3) / 1e9
         roof = {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(ach / peak, 4), "traffic": None,
                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}, burst)",
                 "algorithmic_bytes_per_launch": int(algo_bytes),
-                "l2_fifo_bytes_per_launch": int(4.0 * (nr - 1) / nr * S * nr)}
+                "dram_algorithmic_bytes_per_launch": int(5.0 * (nr - 1) / nr * S * nr)}
     tr = os.environ.get("RESCCL_BENCH_TRAFFIC")
     if tr:
         roof["traffic"] = float(tr)

@@ -134,6 +134,13 @@ rescclResult_t rescclSetActiveAlgorithm(rescclComm_t comm, rescclAlgo_t algo);
  * connection groups, TB counts, layout).  Same size protocol as rescclCommGetHandle. */
 rescclResult_t rescclGetPlanInfo(rescclAlgo_t algo, char* json, size_t* len);
 
+/* TB utilisation of the last launch of `algo` (§5.4): per lane
+ * ("TB" in the paper's count) its lifetime and the time it spent busy-waiting on
+ * dependencies, payload or credit; plus Comm Time = 1 - mean idle ratio, Avg Idle,
+ * Max Idle (Table 3's columns).  Requires the algorithm loaded with trace=1 (or
+ * RESCCL_TRACE=1) and the launch finished (synchronise the stream first). */
+rescclResult_t rescclGetTbUtilization(rescclAlgo_t algo, char* json, size_t* len);
+
 /* ------------------------------------------------------------------ collectives */
 
 /* out_r[i] = sum_k in_k[i].  sendbuf/recvbuf: count elements each. */

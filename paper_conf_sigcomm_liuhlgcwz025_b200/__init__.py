@@ -42,7 +42,8 @@ EXPORTS = [
     "rescclGetErrorString", "rescclGetLastError", "rescclGetVersion", "rescclCommCreate",
     "rescclCommGetHandle", "rescclCommConnect", "rescclCommInit", "rescclCommInitAll",
     "rescclCommDestroy", "rescclCommRank", "rescclCommCount", "rescclCommGetAsyncError",
-    "rescclLoadAlgorithm", "rescclSetActiveAlgorithm", "rescclGetPlanInfo", "rescclAllReduce",
+    "rescclLoadAlgorithm", "rescclSetActiveAlgorithm", "rescclGetPlanInfo", "rescclGetTbUtilization",
+    "rescclAllReduce",
     "rescclAllGather", "rescclReduceScatter", "rescclGenerateIr", "rescclPlanIr",
     "rescclCodegenIr", "rescclCompileIr", "rescclCheckDeadlock",
 ]
@@ -64,6 +65,7 @@ _SIGS = {
     "rescclLoadAlgorithm": (_i, [_vp, _c.c_char_p, _c.POINTER(_vp)]),
     "rescclSetActiveAlgorithm": (_i, [_vp, _vp]),
     "rescclGetPlanInfo": (_i, [_vp, _c.c_char_p, _c.POINTER(_sz)]),
+    "rescclGetTbUtilization": (_i, [_vp, _c.c_char_p, _c.POINTER(_sz)]),
     "rescclAllReduce": (_i, [_vp, _vp, _sz, _i, _i, _vp, _vp]),
     "rescclAllGather": (_i, [_vp, _vp, _sz, _i, _vp, _vp]),
     "rescclReduceScatter": (_i, [_vp, _vp, _sz, _i, _i, _vp, _vp]),
@@ -183,6 +185,14 @@ def rescclGetPlanInfo(algo: int) -> dict:
     _check(_lib.rescclGetPlanInfo(algo, None, _c.byref(n)), "rescclGetPlanInfo")
     buf = _c.create_string_buffer(n.value)
     _check(_lib.rescclGetPlanInfo(algo, buf, _c.byref(n)), "rescclGetPlanInfo")
+    return json.loads(buf.value.decode())
+
+
+def rescclGetTbUtilization(algo: int) -> dict:
+    n = _sz(0)
+    _check(_lib.rescclGetTbUtilization(algo, None, _c.byref(n)), "rescclGetTbUtilization")
+    buf = _c.create_string_buffer(n.value)
+    _check(_lib.rescclGetTbUtilization(algo, buf, _c.byref(n)), "rescclGetTbUtilization")
     return json.loads(buf.value.decode())
 
 

@@ -49,6 +49,7 @@ struct KArgs {
   int block_base;
   int* err;
   unsigned long long timeout_ns;
+  unsigned long long* trace;
 };
 
 thread_local std::string g_last_error;
@@ -126,8 +127,9 @@ struct Options {
   bool fuse = true;
   int tb_budget = 0;
   int tma = 1;
-  int tma_tile = 16384;
+  int tma_tile = 12288;   // r01 sweep: 12 KiB x 4 stages (192 KiB smem per CTA) is best
   int tma_stages = 4;
+  int trace = 0;
 };
 
 std::map<std::string, std::string> parse_kv(const char* s) {
@@ -164,6 +166,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "tma") o.tma = (int)to_long(v, k);
   else if (k == "tmatile") o.tma_tile = (int)to_long(v, k);
   else if (k == "tmastages") o.tma_stages = (int)to_long(v, k);
+  else if (k == "trace") o.trace = (int)to_long(v, k);
   else if (k == "linkmodel") {
     if (v == "pair") o.model = LinkModel::Pair;
     else if (v == "port") o.model = LinkModel::Port;
@@ -179,7 +182,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -188,8 +191,8 @@ Options make_options(const Ir& ir, const char* extra) {
   if (o.chunk_bytes < 256 || o.chunk_bytes > (1ll << 30)) fail(rescclInvalidArgument, "chunkbytes out of range");
   if (o.nwarps < 2 || o.nwarps > 32 || o.nwarps % 2) fail(rescclInvalidArgument, "nwarps must be even, 2..32");
   if (o.tma_tile < 1024 || o.tma_tile % 128 || o.tma_stages < 1 || o.tma_stages > 8 ||
-      2 * o.tma_tile * o.tma_stages > 200 * 1024)
-    fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 2*tile*stages <= 200 KiB");
+      4 * o.tma_tile * o.tma_stages > 200 * 1024)
+    fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 4*tile*stages <= 200 KiB");
   return o;
 }
 
@@ -288,6 +291,10 @@ struct AlgoShared {
   unsigned long long mb_cum = 0;       // virtual group: one counter for all ranks
   std::map<std::string, Kern> kernels;  // key: dtype/op/ranks/scope
   std::vector<char*> region;           // virtual group: per-rank plan region (one allocation)
+  unsigned long long* trace_host = nullptr;  // RESCCL_TRACE buffer (host-mapped)
+  unsigned long long* trace_dev = nullptr;
+  int trace_blocks = 0;                // blocks covered by the last traced launch
+  int trace_block_base = 0;
   char* region_alloc = nullptr;
   int64_t region_off = 0;              // multi-process: offset inside the arena
 };
@@ -410,6 +417,7 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.tma = a.opt.tma;
   co.tma_tile = a.opt.tma_tile;
   co.tma_stages = a.opt.tma_stages;
+  co.trace = a.opt.trace;
   std::string src = codegen(a.plan, a.lay, co);
   if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
     if (FILE* f = fopen((std::string(dump) + "_" + a.ir.name + "_" + coll_name(a.ir.coll) + ".cu").c_str(), "w")) {
@@ -512,6 +520,20 @@ void fill_geometry(KArgs& ka, const Geometry& g, size_t count) {
   ka.n_mb = g.n_mb;
 }
 
+unsigned long long* trace_buffer(AlgoShared& a, int blocks, int block_base) {
+  if (!a.opt.trace) return nullptr;
+  if (!a.trace_host) {
+    size_t bytes = (size_t)a.lay.total_pairs * a.opt.instances * 2 * 4 * sizeof(unsigned long long);
+    cuda_check(cudaHostAlloc((void**)&a.trace_host, bytes, cudaHostAllocMapped | cudaHostAllocPortable),
+               "cudaHostAlloc(trace)");
+    memset(a.trace_host, 0, bytes);
+    cuda_check(cudaHostGetDevicePointer((void**)&a.trace_dev, a.trace_host, 0), "cudaHostGetDevicePointer");
+  }
+  a.trace_blocks = blocks;
+  a.trace_block_base = block_base;
+  return a.trace_dev;
+}
+
 // multi-process / multi-device path: this rank alone
 void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const void* send, void* recv,
                  cudaStream_t s) {
@@ -533,6 +555,7 @@ void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const vo
   ka.block_base = a.lay.pair_start[comm->rank] * a.opt.instances;
   ka.err = comm->err_dev;
   ka.timeout_ns = timeout_ns();
+  ka.trace = trace_buffer(a, a.lay.ctas[comm->rank] * a.opt.instances, ka.block_base);
   Kern& k = get_kernel(a, c.dt, c.op, comm->rank, comm->rank + 1, false);
   launch(k, a.lay.ctas[comm->rank] * a.opt.instances, 32 * a.opt.nwarps, ka, s);
   algo->mb_cum += (unsigned long long)g.n_mb;
@@ -561,6 +584,7 @@ void group_launch(Group* G, Pending& p) {
   ka.block_base = 0;
   ka.err = G->err_dev;
   ka.timeout_ns = timeout_ns();
+  ka.trace = trace_buffer(a, a.lay.total_pairs * a.opt.instances, 0);
   Kern& k = get_kernel(a, c.dt, c.op, 0, G->nranks, true);
   cudaStream_t ls = p.streams.back();
   // order the launch after every caller's stream, and every caller's stream after it
@@ -971,6 +995,47 @@ rescclResult_t rescclGetPlanInfo(rescclAlgo_t algo, char* json, size_t* len) {
   API_END
 }
 
+rescclResult_t rescclGetTbUtilization(rescclAlgo_t algo, char* json, size_t* len) {
+  API_BEGIN
+  if (!algo) fail(rescclInvalidArgument, "algo is NULL");
+  AlgoShared& a = *algo->s;
+  if (!a.opt.trace || !a.trace_host) fail(rescclInvalidUsage, "no trace: load with trace=1 (RESCCL_TRACE=1) and run");
+  std::ostringstream o;
+  o << "{\"lanes\":[";
+  double sum_idle = 0, max_idle = 0;
+  int n = 0;
+  unsigned long long t_min = ~0ull, t_max = 0;
+  bool first = true;
+  for (int b = 0; b < a.trace_blocks; ++b) {
+    int g = b + a.trace_block_base;
+    int pair = g / a.opt.instances, inst = g % a.opt.instances;
+    int rank = 0;
+    while (rank + 1 < (int)a.lay.pair_start.size() && a.lay.pair_start[rank + 1] <= pair) ++rank;
+    int cta = pair - a.lay.pair_start[rank];
+    for (int lane = 0; lane < 2; ++lane) {
+      volatile unsigned long long* tr = a.trace_host + 4 * (2 * (size_t)b + lane);
+      if (tr[3] == 0 || tr[1] <= tr[0]) continue;
+      double life = (double)(tr[1] - tr[0]);
+      double idle = (double)tr[2] / life;
+      if (idle > 1) idle = 1;
+      sum_idle += idle;
+      max_idle = std::max(max_idle, idle);
+      ++n;
+      t_min = std::min(t_min, (unsigned long long)tr[0]);
+      t_max = std::max(t_max, (unsigned long long)tr[1]);
+      o << (first ? "" : ",") << "[" << rank << "," << cta << "," << inst << "," << lane << "," << (tr[1] - tr[0])
+        << "," << tr[2] << "," << tr[3] << "]";
+      first = false;
+    }
+  }
+  double avg = n ? sum_idle / n : 0;
+  o << "],\"fields\":[\"rank\",\"cta\",\"instance\",\"lane\",\"lifetime_ns\",\"wait_ns\",\"prims\"]"
+    << ",\"tbs\":" << n << ",\"comm_time\":" << (1 - avg) << ",\"avg_idle\":" << avg
+    << ",\"max_idle\":" << max_idle << ",\"span_ns\":" << (n ? t_max - t_min : 0) << "}";
+  write_out(o.str(), json, len);
+  API_END
+}
+
 rescclResult_t rescclAllReduce(const void* sendbuf, void* recvbuf, size_t count, rescclDataType_t dtype,
                                rescclRedOp_t op, rescclComm_t comm, void* stream) {
   API_BEGIN
@@ -1031,6 +1096,7 @@ rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo
   co.tma = o.tma;
   co.tma_tile = o.tma_tile;
   co.tma_stages = o.tma_stages;
+  co.trace = o.trace;
   write_out(codegen(p, L, co), src, len);
   API_END
 }
@@ -1048,6 +1114,7 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
   co.tma = o.tma;
   co.tma_tile = o.tma_tile;
   co.tma_stages = o.tma_stages;
+  co.trace = o.trace;
   co.gpu_scope = true;
   auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, true);
   if (cubin_bytes) *cubin_bytes = cub.size();

@@ -30,6 +30,9 @@
 #ifndef RESCCL_TMA
 #define RESCCL_TMA 1
 #endif
+#ifndef RESCCL_TRACE
+#define RESCCL_TRACE 0
+#endif
 
 namespace rdev {
 
@@ -52,6 +55,7 @@ struct KArgs {
   int block_base;                     // global block id of blockIdx.x == 0
   int* err;                           // host-mapped error word
   u64 timeout_ns;
+  u64* trace;                         // RESCCL_TRACE: 4 x u64 per (block, lane), host-mapped
 };
 
 enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16 };
@@ -132,6 +136,43 @@ __device__ __forceinline__ void mbar_wait(u32 bar, u32 parity) {
       "{\n.reg .pred p;\nWAIT_%=:\n"
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
       "@!p bra WAIT_%=;\n}\n" ::"r"(bar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ bool mbar_test(u32 bar, u32 parity) {
+  u32 ok;
+  asm volatile(
+      "{\n.reg .pred p;\n"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      "selp.u32 %0, 1, 0, p;\n}\n" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_arrive(u32 bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+// wait until at most n bulk groups are pending (n must be an immediate)
+__device__ __forceinline__ void tma_wait_n(u32 n) {
+  switch (n) {
+    case 1: asm volatile("cp.async.bulk.wait_group 1;" ::: "memory"); break;
+    case 2: asm volatile("cp.async.bulk.wait_group 2;" ::: "memory"); break;
+    case 3: asm volatile("cp.async.bulk.wait_group 3;" ::: "memory"); break;
+    case 4: asm volatile("cp.async.bulk.wait_group 4;" ::: "memory"); break;
+    case 5: asm volatile("cp.async.bulk.wait_group 5;" ::: "memory"); break;
+    case 6: asm volatile("cp.async.bulk.wait_group 6;" ::: "memory"); break;
+    case 7: asm volatile("cp.async.bulk.wait_group 7;" ::: "memory"); break;
+    default: asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); break;
+  }
+}
+__device__ __forceinline__ void tma_wait_read_n(u32 n) {
+  switch (n) {
+    case 1: asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); break;
+    case 2: asm volatile("cp.async.bulk.wait_group.read 2;" ::: "memory"); break;
+    case 3: asm volatile("cp.async.bulk.wait_group.read 3;" ::: "memory"); break;
+    case 4: asm volatile("cp.async.bulk.wait_group.read 4;" ::: "memory"); break;
+    case 5: asm volatile("cp.async.bulk.wait_group.read 5;" ::: "memory"); break;
+    case 6: asm volatile("cp.async.bulk.wait_group.read 6;" ::: "memory"); break;
+    case 7: asm volatile("cp.async.bulk.wait_group.read 7;" ::: "memory"); break;
+    default: asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); break;
+  }
 }
 __device__ __forceinline__ void tma_load(u32 dst_smem, const void* src, u32 bytes, u32 bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
@@ -315,15 +356,20 @@ struct Lane {
   char* self;       // this rank's plan region
   int rank, inst, bar, nthreads, tid;
   volatile int* abort_flag;  // shared memory, per lane
-  char* stage;               // this lane's TMA staging buffer (RESCCL_TMA_STAGES tiles)
-  u32 mbar;                  // shared address of this lane's RESCCL_TMA_STAGES mbarriers
-  u32 tma_seq;               // tiles loaded so far (leader only): stage = seq % S, parity = (seq / S) & 1
+  char* stage;               // this lane's TMA staging: RESCCL_TMA_STAGES x (A tile, B tile)
+  u32 full;                  // shared address of the "tile loaded" mbarriers (one per stage)
+  u32 comp;                  // shared address of the "tile combined" mbarriers (one per stage)
+  u32 tseq;                  // tiles streamed so far by this lane: stage = tseq % S, parity = tseq / S
+  u32 comp_use[RESCCL_TMA_STAGES];  // leader: completed phases of each comp barrier
+  volatile u32* issued;      // shared: tiles the leader has issued (combine warps must not test a
+                             // stage's parity before its tile is issued: no ABA on phases)
+  u64 wait_ns;               // RESCCL_TRACE: leader time spent waiting (idle ratio, Table 3)
 
   __device__ __forceinline__ void sync() const {
     asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(nthreads) : "memory");
   }
   // leader only: spin until *p >= target; false on timeout (error word set)
-  __device__ bool wait_ge(const u64* p, u64 target) const {
+  __device__ bool wait_ge(const u64* p, u64 target) {
     if (ld_acquire(p) >= target) return true;
     u64 t0 = globaltimer();
     u32 spins = 0;
@@ -334,6 +380,9 @@ struct Lane {
         return false;
       }
     }
+#if RESCCL_TRACE
+    wait_ns += globaltimer() - t0;
+#endif
     return true;
   }
 };
@@ -358,41 +407,6 @@ __device__ __forceinline__ char* buf_ptr(const KArgs& a, int rank, int buf) {
   return buf == BufSend ? (char*)a.sendbuf[rank] : (buf == BufRecv ? a.recvbuf[rank] : a.scratch[rank]);
 }
 
-// Leader-only: copy `bytes` (multiple of 16; 16-byte aligned pointers) from S to D1
-// and/or D2 through the lane's shared-memory stages.
-__device__ __noinline__ void tma_copy(Lane& L, const char* S, char* D1, char* D2, i64 bytes) {
-  const int NS = RESCCL_TMA_STAGES;
-  const i64 TB = RESCCL_TMA_TILE;
-  const i64 ntiles = (bytes + TB - 1) / TB;
-  const u32 sbase = smem_u32(L.stage);
-  const u32 base = L.tma_seq;
-  auto issue = [&](i64 t) {
-    const u32 k = base + (u32)t;
-    const u32 st = k % NS;
-    const i64 off = t * TB;
-    const u32 nb = (u32)((bytes - off) < TB ? (bytes - off) : TB);
-    mbar_expect_tx(L.mbar + 8 * st, nb);
-    tma_load(sbase + st * (u32)TB, S + off, nb, L.mbar + 8 * st);
-  };
-  for (i64 t = 0; t < ntiles && t < NS; ++t) issue(t);
-  for (i64 t = 0; t < ntiles; ++t) {
-    const u32 k = base + (u32)t;
-    const u32 st = k % NS;
-    const i64 off = t * TB;
-    const u32 nb = (u32)((bytes - off) < TB ? (bytes - off) : TB);
-    mbar_wait(L.mbar + 8 * st, (k / NS) & 1);
-    if (D1) tma_store(D1 + off, sbase + st * (u32)TB, nb);
-    if (D2) tma_store(D2 + off, sbase + st * (u32)TB, nb);
-    tma_commit();
-    if (t + NS < ntiles) {
-      tma_wait_read0();
-      issue(t + NS);
-    }
-  }
-  tma_wait_all();
-  L.tma_seq = base + (u32)ntiles;
-}
-
 // One primitive of the schedule: constants emitted by the kernel generator as a
 // literal.  Offsets are bytes inside the plan region of the named rank's arena, for
 // instance 0 (instance i adds i * K * SLOT, i * FLAGSTRIDE or i * 128).
@@ -409,37 +423,61 @@ struct PrimDesc {
 
 // Layout constants shared by every primitive of a plan (emitted by the generator):
 //   RESCCL_K, RESCCL_I, RESCCL_SLOT, RESCCL_FLAGSTRIDE, RESCCL_COLL
-template <class T, int OP, int F>
-__device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
+struct PrimPtrs {
+  const char* A;     // local operand base (chunk start)
+  char* D1;          // local store target base (chunk start)
+  char* in_data;     // incoming FIFO slots (this instance)
+  u64* in_flag;
+  u64* in_cred;      // credit counter in the sender's arena
+  char* out_data;    // outgoing FIFO slots in the receiver's arena
+  u64* out_flag;
+  u64* out_cred;     // credit counter the receiver writes back (own arena)
+  u64* ctr;
+  i64 len;           // chunk length (elements)
+};
+
+__device__ __forceinline__ void slice_of(const KArgs& a, i64 len, int j, int inst, i64& lo, i64& hi) {
+  lo = (i64)j * a.M + (i64)inst * a.Mi;
+  hi = lo + a.Mi;
+  if (hi > (i64)(j + 1) * a.M) hi = (i64)(j + 1) * a.M;
+  if (hi > len) hi = len;
+  if (lo > hi) lo = hi;
+}
+
+template <int F>
+__device__ __forceinline__ void post_mb(const KArgs& a, const PrimDesc& d, const PrimPtrs& p, int j) {
+  const u64 mb_base = a.mb_base;
+  const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
+  const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
+  fence_release();
+  if (F & kSend) st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);
+  if (F & kRecv) st_relaxed(p.in_cred, in_seq + 1);
+  if (d.ctr >= 0) st_relaxed(p.ctr, mb_base + j + 1);
+}
+
+// Non-blocking readiness of micro-batch j: local dependencies, payload, credit.
+template <int F>
+__device__ __forceinline__ bool mb_ready(const Lane& L, const PrimDesc& d, const PrimPtrs& p, int j) {
   const KArgs& a = *L.a;
-  const int c = d.chunk;
-  const i64 len = chunk_len<RESCCL_COLL>(a, c);
-  const char* A = nullptr;
-  char* D1 = nullptr;
-  if ((F & kCopy) || (F & kReduce) || !(F & kRecv))
-    A = buf_ptr(a, L.rank, d.src_buf) + chunk_off<RESCCL_COLL>(d.src_buf, c, a.C) * T::kSize;
-  if ((F & kCopy) || (F & kStore))
-    D1 = buf_ptr(a, L.rank, d.dst_buf) + chunk_off<RESCCL_COLL>(d.dst_buf, c, a.C) * T::kSize;
-  if (F & kCopy) {
-    if (A == D1) return true;  // in-place: own chunk already in place
-    for (int j = 0; j < a.n_mb; ++j) {
-      i64 lo = (i64)j * a.M + (i64)L.inst * a.Mi;
-      i64 hi = lo + a.Mi;
-      if (hi > (i64)(j + 1) * a.M) hi = (i64)(j + 1) * a.M;
-      if (hi > len) hi = len;
-      if (lo > hi) lo = hi;
-      move<T, OP, kCopy, 4>(hi - lo, A + lo * T::kSize, nullptr, D1 + lo * T::kSize, nullptr, L.tid, L.nthreads);
-    }
-    return true;
+  const u64 mb_base = a.mb_base;
+  for (int k = 0; k < d.ndeps; ++k)
+    if (ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) < mb_base + j + 1) return false;
+  if (F & kRecv) {
+    const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
+    if (ld_acquire(p.in_flag + (in_seq % RESCCL_K)) < in_seq + 1) return false;
   }
-  char* in_data = L.self + d.in_data + (i64)L.inst * RESCCL_K * RESCCL_SLOT;
-  u64* in_flag = at(L.self, d.in_flag + (i64)L.inst * RESCCL_FLAGSTRIDE);
-  u64* in_cred = (F & kRecv) ? at(a.arena[d.in_peer], d.in_cred + (i64)L.inst * 128) : nullptr;
-  char* peer = (F & kSend) ? a.arena[d.out_peer] : nullptr;
-  char* out_data = (F & kSend) ? peer + d.out_data + (i64)L.inst * RESCCL_K * RESCCL_SLOT : nullptr;
-  u64* out_flag = (F & kSend) ? at(peer, d.out_flag + (i64)L.inst * RESCCL_FLAGSTRIDE) : nullptr;
-  u64* out_cred = at(L.self, d.out_cred + (i64)L.inst * 128);
-  u64* ctr = at(L.self, d.ctr + (i64)L.inst * 128);
+  if (F & kSend) {
+    const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
+    if (out_seq + 1 > (u64)RESCCL_K && ld_acquire(p.out_cred) < out_seq + 1 - RESCCL_K) return false;
+  }
+  return true;
+}
+
+// Blocking per-micro-batch path (all lane threads; 16-byte LD/ST): used for misaligned
+// buffers and when the TMA pipeline is disabled.
+template <class T, int OP, int F>
+__device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
+  const KArgs& a = *L.a;
   const u64 mb_base = a.mb_base;
   for (int j = 0; j < a.n_mb; ++j) {
     const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
@@ -448,47 +486,274 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
       bool ok = true;
       for (int k = 0; k < d.ndeps && ok; ++k)
         ok = L.wait_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), mb_base + j + 1);
-      if (ok && (F & kRecv)) ok = L.wait_ge(in_flag + (in_seq % RESCCL_K), in_seq + 1);
-      if (ok && (F & kSend) && out_seq + 1 > (u64)RESCCL_K) ok = L.wait_ge(out_cred, out_seq + 1 - RESCCL_K);
+      if (ok && (F & kRecv)) ok = L.wait_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1);
+      if (ok && (F & kSend) && out_seq + 1 > (u64)RESCCL_K) ok = L.wait_ge(p.out_cred, out_seq + 1 - RESCCL_K);
       if (!ok) *L.abort_flag = 1;
     }
     L.sync();
     if (*L.abort_flag) return false;
-    i64 lo = (i64)j * a.M + (i64)L.inst * a.Mi;
-    i64 hi = lo + a.Mi;
-    if (hi > (i64)(j + 1) * a.M) hi = (i64)(j + 1) * a.M;
-    if (hi > len) hi = len;
-    if (lo > hi) lo = hi;
-    const char* Aj = A ? A + lo * T::kSize : nullptr;
-    char* D1j = D1 ? D1 + lo * T::kSize : nullptr;
-    const char* Bj = (F & kRecv) ? in_data + (in_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
-    char* D2j = (F & kSend) ? out_data + (out_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
-#if RESCCL_TMA
-    if (!(F & kReduce)) {
-      // pure data movement: bulk copy the 16-byte-aligned body, threads do the tail
-      const char* Sj = (F & kRecv) ? Bj : Aj;
-      const unsigned long long al = (unsigned long long)Sj | (unsigned long long)D1j | (unsigned long long)D2j;
-      const i64 nb = (al & 15) ? 0 : (((hi - lo) * T::kSize) & ~(i64)15);
-      if (L.tid == 0 && nb > 0) {
-        fence_proxy_async();
-        tma_copy(L, Sj, D1j, D2j, nb);
-        fence_proxy_async();
-      }
-      const i64 e0 = nb / T::kSize;
-      move<T, OP, F, 4>(hi - lo - e0, Aj ? Aj + nb : nullptr, Bj ? Bj + nb : nullptr, D1j ? D1j + nb : nullptr,
-                        D2j ? D2j + nb : nullptr, L.tid, L.nthreads);
-    } else
-#endif
-      move<T, OP, F, 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
+    i64 lo, hi;
+    slice_of(a, p.len, j, L.inst, lo, hi);
+    const char* Aj = p.A ? p.A + lo * T::kSize : nullptr;
+    char* D1j = p.D1 ? p.D1 + lo * T::kSize : nullptr;
+    const char* Bj = (F & kRecv) ? p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
+    char* D2j = (F & kSend) ? p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
+    move<T, OP, F, 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
     L.sync();
-    if (L.tid == 0) {
-      fence_release();
-      if (F & kSend) st_relaxed(out_flag + (out_seq % RESCCL_K), out_seq + 1);
-      if (F & kRecv) st_relaxed(in_cred, in_seq + 1);
-      if (d.ctr >= 0) st_relaxed(ctr, mb_base + j + 1);
-    }
+    if (L.tid == 0) post_mb<F>(a, d, p, j);
   }
   return true;
+}
+
+// Number of TMA tiles of micro-batch j (16-byte-aligned body only).  A stage holds one
+// reduce tile (A and B halves of RESCCL_TMA_TILE bytes) or one copy tile of twice that.
+template <int F>
+__device__ __forceinline__ i64 tile_bytes() { return (F & kReduce) ? RESCCL_TMA_TILE : 2 * RESCCL_TMA_TILE; }
+template <int F>
+__device__ __forceinline__ u32 mb_tiles(const KArgs& a, i64 len, int j, int inst, int esz, i64& lo, i64& nb) {
+  i64 hi;
+  slice_of(a, len, j, inst, lo, hi);
+  nb = ((hi - lo) * esz) & ~(i64)15;
+  return (u32)((nb + tile_bytes<F>() - 1) / tile_bytes<F>());
+}
+
+// TMA pipeline, leader thread: a non-blocking event loop that (1) confirms the
+// readiness of the next micro-batch, (2) streams its tiles into the stage ring with
+// cp.async.bulk, (3) stores tiles whose data is loaded (copy) or combined (reduce) to
+// the local buffer and/or the peer FIFO, (4) posts a micro-batch once all its stores
+// completed.  It never blocks on a remote condition while it holds unposted work, so
+// the pipeline adds no wait edge beyond those of the blocking model (deadlock freedom
+// carries over from the plan check).
+template <class T, int OP, int F>
+__device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
+  const KArgs& a = *L.a;
+  const int NS = RESCCL_TMA_STAGES;
+  const i64 TB = tile_bytes<F>();
+  const int nmb = a.n_mb;
+  const u32 k0 = L.tseq;
+  const u32 sbase = smem_u32(L.stage);
+  const u64 mb_base = a.mb_base;
+  int rj = 0;                 // micro-batches whose readiness is confirmed
+  int lj = 0;                 // load cursor (micro-batch, tile)
+  u32 lt = 0;
+  u32 issued = 0, stored = 0; // tiles
+  int sj = 0;                 // store cursor
+  u32 st = 0;
+  int pj = 0;                 // next micro-batch to post
+  i64 lo_l = 0, nb_l = 0, lo_s = 0, nb_s = 0, lo_p = 0, nb_p = 0;
+  u32 T_l = mb_tiles<F>(a, p.len, 0, L.inst, T::kSize, lo_l, nb_l);
+  u32 T_s = T_l;
+  lo_s = lo_l;
+  nb_s = nb_l;
+  u32 T_p = T_l;
+  lo_p = lo_l;
+  nb_p = nb_l;
+  u32 gp_end = T_l;           // tiles through micro-batch pj
+  u64 t_idle = 0;
+  u32 spins = 0;
+  while (pj < nmb) {
+    bool prog = false;
+    // (1) readiness of the micro-batch the load cursor needs
+    if (rj < nmb && rj == lj && mb_ready<F>(L, d, p, rj)) {
+      fence_proxy_async();  // generic-proxy data (acquired) -> async-proxy reads
+      ++rj;
+      prog = true;
+    }
+    // (2) loads
+    while (lj < rj) {
+      if (lt >= T_l) {
+        ++lj;
+        lt = 0;
+        if (lj < nmb) T_l = mb_tiles<F>(a, p.len, lj, L.inst, T::kSize, lo_l, nb_l);
+        continue;
+      }
+      if (issued - stored >= (u32)NS) break;
+      if (issued >= (u32)NS) tma_wait_read_n(stored - 1 - (issued - NS));  // stage's last store read smem
+      const u32 k = k0 + issued;
+      const u32 s = k % NS;
+      const i64 off = (i64)lt * TB;
+      const u32 nb = (u32)((nb_l - off) < TB ? (nb_l - off) : TB);
+      const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
+      if (F & kReduce) {
+        const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + lj;
+        mbar_expect_tx(L.full + 8 * s, 2 * nb);
+        tma_load(sa, p.A + lo_l * T::kSize + off, nb, L.full + 8 * s);
+        tma_load(sa + (u32)RESCCL_TMA_TILE, p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off, nb, L.full + 8 * s);
+      } else {
+        const char* src;
+        if (F & kRecv) {
+          const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + lj;
+          src = p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off;
+        } else {
+          src = p.A + lo_l * T::kSize + off;
+        }
+        mbar_expect_tx(L.full + 8 * s, nb);
+        tma_load(sa, src, nb, L.full + 8 * s);
+      }
+      ++issued;
+      ++lt;
+      if (F & kReduce) *L.issued = k0 + issued;
+      prog = true;
+    }
+    // (3) stores
+    while (stored < issued) {
+      const u32 k = k0 + stored;
+      const u32 s = k % NS;
+      const bool ok = (F & kReduce) ? mbar_test(L.comp + 8 * s, L.comp_use[s] & 1)
+                                    : mbar_test(L.full + 8 * s, (k / NS) & 1);
+      if (!ok) break;
+      while (st >= T_s) {
+        ++sj;
+        st = 0;
+        T_s = mb_tiles<F>(a, p.len, sj, L.inst, T::kSize, lo_s, nb_s);
+      }
+      const i64 off = (i64)st * TB;
+      const u32 nb = (u32)((nb_s - off) < TB ? (nb_s - off) : TB);
+      const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
+      if (F & kStore) tma_store(p.D1 + lo_s * T::kSize + off, sa, nb);
+      if (F & kSend) {
+        const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + sj;
+        tma_store(p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + off, sa, nb);
+      }
+      tma_commit();
+      if (F & kReduce) L.comp_use[s]++;
+      ++stored;
+      ++st;
+      prog = true;
+    }
+    // (4) post
+    if (pj < rj && stored >= gp_end) {
+      tma_wait_n(stored - gp_end);
+      // unaligned tail (< 16 bytes) of this micro-batch: scalar, by the leader
+      i64 lo_h, hi_h;
+      slice_of(a, p.len, pj, L.inst, lo_h, hi_h);
+      const i64 e0 = lo_h + nb_p / T::kSize;
+      if (e0 < hi_h) {
+        const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + pj;
+        const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + pj;
+        const char* Bj = (F & kRecv) ? p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + nb_p : nullptr;
+        char* D2j = (F & kSend) ? p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + nb_p : nullptr;
+        for (i64 e = 0; e < hi_h - e0; ++e)
+          elem_move<T, OP>(F, p.A ? p.A + e0 * T::kSize : nullptr, Bj, p.D1 ? p.D1 + e0 * T::kSize : nullptr, D2j, e);
+      }
+      fence_proxy_async();
+      post_mb<F>(a, d, p, pj);
+      ++pj;
+      if (pj < nmb) {
+        T_p = mb_tiles<F>(a, p.len, pj, L.inst, T::kSize, lo_p, nb_p);
+        gp_end += T_p;
+      }
+      prog = true;
+    }
+    if (prog) {
+#if RESCCL_TRACE
+      if (t_idle) L.wait_ns += globaltimer() - t_idle;
+#endif
+      spins = 0;
+      t_idle = 0;
+    } else {
+#if RESCCL_TRACE
+      if (t_idle == 0) t_idle = globaltimer();
+#endif
+      if (++spins > 32) nanosleep_(20);
+      if ((spins & 255) == 0) {
+        const u64 now = globaltimer();
+        if (t_idle == 0) t_idle = now;
+        else if (now - t_idle > a.timeout_ns) {
+          atomicCAS(a.err, 0, kErrTimeout);
+          *L.abort_flag = 1;
+          return false;
+        }
+      }
+    }
+  }
+#if RESCCL_TRACE
+  if (t_idle) L.wait_ns += globaltimer() - t_idle;
+#endif
+  L.tseq = k0 + issued;
+  return true;
+}
+
+// TMA pipeline, combine warps (reduce primitives): tile k of the lane's stream is
+// combined in shared memory as soon as its A and B tiles land.
+template <class T, int OP, int F>
+__device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const PrimPtrs& p, int ctid, int nct) {
+  const KArgs& a = *L.a;
+  const int NS = RESCCL_TMA_STAGES;
+  const i64 TB = RESCCL_TMA_TILE;  // reduce tiles only
+  u32 k = L.tseq;
+  for (int j = 0; j < a.n_mb; ++j) {
+    i64 lo, nbj;
+    const u32 ntl = mb_tiles<F>(a, p.len, j, L.inst, T::kSize, lo, nbj);
+    for (u32 t = 0; t < ntl; ++t, ++k) {
+      const u32 s = k % NS;
+      const i64 off = (i64)t * TB;
+      const int nb = (int)((nbj - off) < TB ? (nbj - off) : TB);
+      u32 spins = 0;
+      while ((int)(*L.issued - k) <= 0) {  // tile k not issued yet
+        if (++spins > 16) nanosleep_(20);
+        if ((spins & 1023) == 0 && *L.abort_flag) return false;
+      }
+      while (!mbar_test(L.full + 8 * s, (k / NS) & 1)) {
+        if (++spins > 16) nanosleep_(20);
+        if ((spins & 1023) == 0 && *L.abort_flag) return false;
+      }
+      V4* av = (V4*)(L.stage + (i64)s * 2 * TB);
+      const V4* bv = (const V4*)(L.stage + (i64)s * 2 * TB + TB);
+      for (int i = ctid; i < nb / 16; i += nct) av[i] = combine_v<T, OP>(av[i], bv[i]);
+      fence_proxy_async_smem();
+      __syncwarp();
+      if ((threadIdx.x & 31) == 0) mbar_arrive(L.comp + 8 * s);
+    }
+  }
+  L.tseq = k;
+  return true;
+}
+
+template <class T, int OP, int F>
+__device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
+  const KArgs& a = *L.a;
+  const int c = d.chunk;
+  PrimPtrs p;
+  p.len = chunk_len<RESCCL_COLL>(a, c);
+  p.A = nullptr;
+  p.D1 = nullptr;
+  if ((F & kCopy) || (F & kReduce) || !(F & kRecv))
+    p.A = buf_ptr(a, L.rank, d.src_buf) + chunk_off<RESCCL_COLL>(d.src_buf, c, a.C) * T::kSize;
+  if ((F & kCopy) || (F & kStore))
+    p.D1 = buf_ptr(a, L.rank, d.dst_buf) + chunk_off<RESCCL_COLL>(d.dst_buf, c, a.C) * T::kSize;
+  if (F & kCopy) {
+    if (p.A == p.D1) return true;  // in-place: own chunk already in place
+    for (int j = 0; j < a.n_mb; ++j) {
+      i64 lo, hi;
+      slice_of(a, p.len, j, L.inst, lo, hi);
+      move<T, OP, kCopy, 4>(hi - lo, p.A + lo * T::kSize, nullptr, p.D1 + lo * T::kSize, nullptr, L.tid, L.nthreads);
+    }
+    return true;
+  }
+  p.in_data = L.self + d.in_data + (i64)L.inst * RESCCL_K * RESCCL_SLOT;
+  p.in_flag = at(L.self, d.in_flag + (i64)L.inst * RESCCL_FLAGSTRIDE);
+  p.in_cred = (F & kRecv) ? at(a.arena[d.in_peer], d.in_cred + (i64)L.inst * 128) : nullptr;
+  char* peer = (F & kSend) ? a.arena[d.out_peer] : nullptr;
+  p.out_data = (F & kSend) ? peer + d.out_data + (i64)L.inst * RESCCL_K * RESCCL_SLOT : nullptr;
+  p.out_flag = (F & kSend) ? at(peer, d.out_flag + (i64)L.inst * RESCCL_FLAGSTRIDE) : nullptr;
+  p.out_cred = at(L.self, d.out_cred + (i64)L.inst * 128);
+  p.ctr = at(L.self, d.ctr + (i64)L.inst * 128);
+#if RESCCL_TMA
+  const unsigned long long al = (unsigned long long)p.A | (unsigned long long)p.D1;
+  if ((al & 15) == 0) {
+    if (L.tid == 0) return pipe_leader<T, OP, F>(L, d, p);
+    if (L.tid < 32) return true;
+    if (F & kReduce) return pipe_compute<T, OP, F>(L, d, p, L.tid - 32, L.nthreads - 32);
+    // combine warps only keep the lane's tile counter in step for copy primitives
+    for (int j = 0; j < a.n_mb; ++j) {
+      i64 lo, nb;
+      L.tseq += mb_tiles<F>(a, p.len, j, L.inst, T::kSize, lo, nb);
+    }
+    return true;
+  }
+#endif
+  return run_sync<T, OP, F>(L, d, p);
 }
 
 }  // namespace rdev

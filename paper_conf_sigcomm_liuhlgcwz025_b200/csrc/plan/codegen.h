@@ -42,12 +42,14 @@ struct CodegenOpts {
   bool gpu_scope = false;        // all ranks on one device (virtual ranks): .gpu-scope flags
   int nwarps = 16;
   int tma = 1;                   // bulk-copy (TMA) data path for non-reducing primitives
-  int tma_tile = 16384;          // bytes per staged tile
+  int tma_tile = 12288;          // bytes per staged tile
   int tma_stages = 4;            // tiles in flight per lane
+  int trace = 0;                 // per-lane lifetime / wait timers (TB utilisation, Table 3)
 };
 
 // dynamic shared memory the generated kernel needs (both lanes' TMA staging)
-inline int codegen_smem_bytes(const CodegenOpts& o) { return o.tma ? 2 * o.tma_stages * o.tma_tile : 0; }
+// (2 lanes x stages x (A tile + B tile))
+inline int codegen_smem_bytes(const CodegenOpts& o) { return o.tma ? 4 * o.tma_stages * o.tma_tile : 0; }
 
 // Device code (without the L0 library text, which the runtime prepends).
 std::string codegen(const Plan& p, const Layout& L, const CodegenOpts& o);
