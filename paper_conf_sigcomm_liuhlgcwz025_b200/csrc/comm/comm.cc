@@ -130,6 +130,8 @@ struct Options {
   int tma_tile = 12288;   // r01 sweep: 12 KiB x 4 stages (192 KiB smem per CTA) is best
   int tma_stages = 4;
   int trace = 0;
+  int l2hint = 1;
+  int prefetch = 2;
 };
 
 std::map<std::string, std::string> parse_kv(const char* s) {
@@ -167,6 +169,8 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "tmatile") o.tma_tile = (int)to_long(v, k);
   else if (k == "tmastages") o.tma_stages = (int)to_long(v, k);
   else if (k == "trace") o.trace = (int)to_long(v, k);
+  else if (k == "l2hint") o.l2hint = (int)to_long(v, k);
+  else if (k == "prefetch") o.prefetch = (int)to_long(v, k);
   else if (k == "linkmodel") {
     if (v == "pair") o.model = LinkModel::Pair;
     else if (v == "port") o.model = LinkModel::Port;
@@ -182,7 +186,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -394,7 +398,7 @@ std::string info_json(const AlgoShared& a) {
   std::string pj = plan_json(a.plan);
   o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
     << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"tma\":" << a.opt.tma
-    << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"linkmodel\":\""
+    << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"l2hint\":" << a.opt.l2hint << ",\"prefetch\":" << a.opt.prefetch << ",\"linkmodel\":\""
     << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
     << ",\"ctas\":[";
   for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];
@@ -418,6 +422,8 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.tma_tile = a.opt.tma_tile;
   co.tma_stages = a.opt.tma_stages;
   co.trace = a.opt.trace;
+  co.l2hint = a.opt.l2hint;
+  co.prefetch = a.opt.prefetch;
   std::string src = codegen(a.plan, a.lay, co);
   if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
     if (FILE* f = fopen((std::string(dump) + "_" + a.ir.name + "_" + coll_name(a.ir.coll) + ".cu").c_str(), "w")) {
@@ -1097,6 +1103,8 @@ rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo
   co.tma_tile = o.tma_tile;
   co.tma_stages = o.tma_stages;
   co.trace = o.trace;
+  co.l2hint = o.l2hint;
+  co.prefetch = o.prefetch;
   write_out(codegen(p, L, co), src, len);
   API_END
 }
@@ -1115,6 +1123,8 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
   co.tma_tile = o.tma_tile;
   co.tma_stages = o.tma_stages;
   co.trace = o.trace;
+  co.l2hint = o.l2hint;
+  co.prefetch = o.prefetch;
   co.gpu_scope = true;
   auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, true);
   if (cubin_bytes) *cubin_bytes = cub.size();

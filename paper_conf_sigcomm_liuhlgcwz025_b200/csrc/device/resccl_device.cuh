@@ -174,13 +174,49 @@ __device__ __forceinline__ void tma_wait_read_n(u32 n) {
     default: asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); break;
   }
 }
-__device__ __forceinline__ void tma_load(u32 dst_smem, const void* src, u32 bytes, u32 bar) {
+// L2 eviction priorities (createpolicy): FIFO slots are written with evict_last so they
+// stay L2-resident between producer and consumer; streamed user data and consumed FIFO
+// payloads use evict_first (RESCCL_L2HINT, default on).
+#ifndef RESCCL_L2HINT
+#define RESCCL_L2HINT 1
+#endif
+__device__ __forceinline__ u64 policy_evict_first() {
+  u64 p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ u64 policy_evict_last() {
+  u64 p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void tma_load(u32 dst_smem, const void* src, u32 bytes, u32 bar, u64 pol) {
+#if RESCCL_L2HINT
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+      ::"r"(dst_smem), "l"(src), "r"(bytes), "r"(bar), "l"(pol) : "memory");
+#else
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                ::"r"(dst_smem), "l"(src), "r"(bytes), "r"(bar) : "memory");
+#endif
 }
-__device__ __forceinline__ void tma_store(void* dst, u32 src_smem, u32 bytes) {
+__device__ __forceinline__ void tma_store(void* dst, u32 src_smem, u32 bytes, u64 pol) {
+#if RESCCL_L2HINT
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;"
+               ::"l"(dst), "r"(src_smem), "r"(bytes), "l"(pol) : "memory");
+#else
   asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src_smem), "r"(bytes)
                : "memory");
+#endif
+}
+#ifndef RESCCL_PREFETCH
+#define RESCCL_PREFETCH 2
+#endif
+// Bulk prefetch of local HBM data into L2 (no shared memory involved).  L2 is the
+// device's point of coherence, so prefetching a slice before its producer finished
+// is safe: later writes update the L2 lines.
+__device__ __forceinline__ void l2_prefetch(const void* p, u32 bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
 }
 __device__ __forceinline__ void tma_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void tma_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
@@ -551,8 +587,22 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   u32 gp_end = T_l;           // tiles through micro-batch pj
   u64 t_idle = 0;
   u32 spins = 0;
+  const u64 pol_first = policy_evict_first();
+  const u64 pol_last = policy_evict_last();
+  int pf = 0;                 // next micro-batch whose local slice gets an L2 prefetch
   while (pj < nmb) {
     bool prog = false;
+#if RESCCL_PREFETCH
+    // (0) keep the local operand of the next RESCCL_PREFETCH micro-batches streaming into L2
+    if (p.A && (F & (kReduce | kRecv)) != kRecv) {
+      while (pf < nmb && pf <= lj + RESCCL_PREFETCH) {
+        i64 lo_f, nb_f;
+        mb_tiles<F>(a, p.len, pf, L.inst, T::kSize, lo_f, nb_f);
+        if (nb_f > 0) l2_prefetch(p.A + lo_f * T::kSize, (u32)nb_f);
+        ++pf;
+      }
+    }
+#endif
     // (1) readiness of the micro-batch the load cursor needs
     if (rj < nmb && rj == lj && mb_ready<F>(L, d, p, rj)) {
       fence_proxy_async();  // generic-proxy data (acquired) -> async-proxy reads
@@ -577,8 +627,9 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       if (F & kReduce) {
         const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + lj;
         mbar_expect_tx(L.full + 8 * s, 2 * nb);
-        tma_load(sa, p.A + lo_l * T::kSize + off, nb, L.full + 8 * s);
-        tma_load(sa + (u32)RESCCL_TMA_TILE, p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off, nb, L.full + 8 * s);
+        tma_load(sa, p.A + lo_l * T::kSize + off, nb, L.full + 8 * s, pol_first);
+        tma_load(sa + (u32)RESCCL_TMA_TILE, p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off, nb,
+                 L.full + 8 * s, pol_first);
       } else {
         const char* src;
         if (F & kRecv) {
@@ -588,7 +639,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
           src = p.A + lo_l * T::kSize + off;
         }
         mbar_expect_tx(L.full + 8 * s, nb);
-        tma_load(sa, src, nb, L.full + 8 * s);
+        tma_load(sa, src, nb, L.full + 8 * s, pol_first);
       }
       ++issued;
       ++lt;
@@ -610,10 +661,10 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       const i64 off = (i64)st * TB;
       const u32 nb = (u32)((nb_s - off) < TB ? (nb_s - off) : TB);
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
-      if (F & kStore) tma_store(p.D1 + lo_s * T::kSize + off, sa, nb);
+      if (F & kStore) tma_store(p.D1 + lo_s * T::kSize + off, sa, nb, pol_first);
       if (F & kSend) {
         const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + sj;
-        tma_store(p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + off, sa, nb);
+        tma_store(p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + off, sa, nb, pol_last);
       }
       tma_commit();
       if (F & kReduce) L.comp_use[s]++;
