@@ -213,10 +213,10 @@ def main():
     S = count * elt
     tdt = getattr(torch, args.dtype)
     # default tuning: fill the SMs at N=1 (8 virtual ranks share one GPU)
-    # default tuning (r01 sweep, profiles/r01_*): 16 instances x 8 virtual ranks = 128 CTAs,
-    # 2 MiB transfer chunks, FIFO depth 2 (keeps the FIFOs L2-resident)
-    inst = args.instances or 16
-    opts = {"instances": inst, "chunkbytes": args.chunk_bytes or (2 << 20), "fifodepth": args.fifo_depth or 2,
+    # default tuning (r01 sweeps, profiles/r01_*): 18 instances x 8 virtual ranks = 144 CTAs
+    # (of 148 SMs), 4 MiB transfer chunks, FIFO depth 2 (FIFOs stay L2-resident)
+    inst = args.instances or 18
+    opts = {"instances": inst, "chunkbytes": args.chunk_bytes or (4 << 20), "fifodepth": args.fifo_depth or 2,
             "nwarps": args.nwarps or None, "tma": None if args.tma < 0 else args.tma}
     text = ir_text(R, args.algo, n, opts)
 

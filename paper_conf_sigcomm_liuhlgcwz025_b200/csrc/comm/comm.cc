@@ -130,8 +130,9 @@ struct Options {
   int tma_tile = 12288;   // r01 sweep: 12 KiB x 4 stages (192 KiB smem per CTA) is best
   int tma_stages = 4;
   int trace = 0;
+  int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
   int l2hint = 1;
-  int prefetch = 2;
+  int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
 };
 
 std::map<std::string, std::string> parse_kv(const char* s) {
@@ -171,6 +172,11 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "trace") o.trace = (int)to_long(v, k);
   else if (k == "l2hint") o.l2hint = (int)to_long(v, k);
   else if (k == "prefetch") o.prefetch = (int)to_long(v, k);
+  else if (k == "sched") {
+    if (v == "hpds") o.sched = 0;
+    else if (v == "rr") o.sched = 1;
+    else fail(rescclInvalidArgument, "sched must be hpds|rr");
+  }
   else if (k == "linkmodel") {
     if (v == "pair") o.model = LinkModel::Pair;
     else if (v == "port") o.model = LinkModel::Port;
@@ -186,7 +192,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -203,9 +209,18 @@ Options make_options(const Ir& ir, const char* extra) {
 // Plan an IR under the options.  A TB budget B picks the link
 // model and the instance count: instances = floor(B / T_min) under the pair model;
 // below T_min the port model (one duplex CTA per rank) with B instances.
+Plan lower_with(const Ir& ir, LinkModel m, const Options& o) {
+  if (o.sched == 1) {
+    Dag d = build_dag(ir);
+    auto pr = round_robin(ir, d, m);
+    return lower(ir, m, o.fuse, &pr);
+  }
+  return lower(ir, m, o.fuse);
+}
+
 Plan make_plan(const Ir& ir, Options& o) {
   if (o.tb_budget > 0) {
-    Plan p = lower(ir, LinkModel::Pair, o.fuse);
+    Plan p = lower_with(ir, LinkModel::Pair, o);
     int tmin = 1;
     for (auto& r : p.ranks) tmin = std::max(tmin, (int)r.ctas.size());
     if (o.tb_budget >= tmin) {
@@ -214,13 +229,13 @@ Plan make_plan(const Ir& ir, Options& o) {
       return p;
     }
     o.model = LinkModel::Port;
-    Plan q = lower(ir, LinkModel::Port, o.fuse);
+    Plan q = lower_with(ir, LinkModel::Port, o);
     int t1 = 1;
     for (auto& r : q.ranks) t1 = std::max(t1, (int)r.ctas.size());
     o.instances = std::max(1, o.tb_budget / t1);
     return q;
   }
-  return lower(ir, o.model, o.fuse);
+  return lower_with(ir, o.model, o);
 }
 
 Plan plan_checked(const Ir& ir, Options& o) {
@@ -398,7 +413,8 @@ std::string info_json(const AlgoShared& a) {
   std::string pj = plan_json(a.plan);
   o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
     << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"tma\":" << a.opt.tma
-    << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"l2hint\":" << a.opt.l2hint << ",\"prefetch\":" << a.opt.prefetch << ",\"linkmodel\":\""
+    << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"l2hint\":" << a.opt.l2hint << ",\"prefetch\":" << a.opt.prefetch << ",\"sched\":\""
+    << (a.opt.sched ? "rr" : "hpds") << "\"" << ",\"linkmodel\":\""
     << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
     << ",\"ctas\":[";
   for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];

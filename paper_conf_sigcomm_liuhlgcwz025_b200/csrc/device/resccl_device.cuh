@@ -210,7 +210,7 @@ __device__ __forceinline__ void tma_store(void* dst, u32 src_smem, u32 bytes, u6
 #endif
 }
 #ifndef RESCCL_PREFETCH
-#define RESCCL_PREFETCH 2
+#define RESCCL_PREFETCH 0
 #endif
 // Bulk prefetch of local HBM data into L2 (no shared memory involved).  L2 is the
 // device's point of coherence, so prefetching a slice before its producer finished

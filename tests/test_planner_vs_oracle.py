@@ -198,3 +198,15 @@ def test_generated_code_has_no_interpreter():
     src = R.rescclCodegenIr(text, "")
     assert src.count("rdev::run<") == 4 * 2 * 6  # 4 ranks x (send + recv) x 2(N-1) steps
     assert "switch (g / RESCCL_I)" in src
+
+
+@pytest.mark.parametrize("name,coll,n,kw", CASES)
+def test_round_robin_plan_matches_oracle(name, coll, n, kw):
+    """RR baseline: C++ sched=rr == oracle hpds.round_robin."""
+    g = _oracle_ir(name, coll, n, kw)
+    js = R.rescclPlanIr(g.to_text(), "sched=rr")
+    edges, _ = dag.build_dag(g)
+    pr = hpds.round_robin(g, edges)
+    tasks = [tuple(t) for t in js["plan"]["tasks"]]
+    assert [[tasks[i] for i in pc] for pc in js["plan"]["Pr"]] == [[tuple(g.transfers[i]) for i in pc] for pc in pr]
+    assert _norm_cpp(js) == _norm_oracle(lower.lower(g, "pair", Pr=pr))

@@ -1,0 +1,98 @@
+"""Measurement sweeps on one B200 (8 virtual ranks), one JSON line per point:
+  c2     ring allreduce / allgather, 1 KiB .. 1 GiB, bf16 / fp32 / int32   (BASELINE configs[1])
+  c3     DBT and HM 2x4 allreduce under a TB budget 1..16                   (configs[2])
+  c4     synthesized allgather / reducescatter, 4..256 MiB, fanout 2/3      (configs[3])
+  f2     HPDS vs round-robin sub-pipelines (Fig. 10b analogue)
+busBW follows nccl-tests: AR 2(N-1)/N, AG/RS (N-1)/N of algBW, S = per-rank buffer
+(AG: total output; RS: total input).  Usage: python tools/sweep.py c2 [c3 c4 f2]"""
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+
+N = 8
+BASE = dict(instances=18, chunkbytes=4 << 20, fifodepth=2)
+ELT = {"bfloat16": 2, "float32": 4, "int32": 4}
+
+
+def measure(name, coll, gopts, opts, S, dtype="bfloat16", iters=10, warm=3):
+    text = R.rescclGenerateIr(name, coll, N, gopts)
+    hdr, rest = text.split("\n", 1)
+    hdr += "".join(f" {k}={v}" for k, v in opts.items())
+    grp = R.VirtualGroup(N, 0)
+    try:
+        grp.load(hdr + "\n" + rest)
+        info = grp.plan_info()
+        elt = ELT[dtype]
+        if coll == "allreduce":
+            cnt = S // elt
+            sn, rn = cnt, cnt
+        elif coll == "allgather":
+            cnt = S // elt // N
+            sn, rn = cnt, cnt * N
+        else:
+            cnt = S // elt // N
+            sn, rn = cnt * N, cnt
+        tdt = getattr(torch, dtype)
+        if tdt.is_floating_point:
+            s = [torch.randn(sn, device="cuda:0").to(tdt) for _ in range(N)]
+        else:
+            s = [torch.randint(-1000, 1000, (sn,), device="cuda:0", dtype=tdt) for _ in range(N)]
+        r = [torch.empty(rn, device="cuda:0", dtype=tdt) for _ in range(N)]
+        f = getattr(grp, coll)
+        for _ in range(warm):
+            f(s, r)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(iters):
+            f(s, r)
+        e1.record()
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1) / iters
+        err = grp.async_error()
+        Sb = (sn if coll != "allgather" else rn) * elt
+        alg = Sb / (ms * 1e-3) / 1e9
+        bus = alg * (2 * (N - 1) / N if coll == "allreduce" else (N - 1) / N)
+        return {"algo": name, "coll": coll, "gopts": gopts, "opts": opts, "dtype": dtype, "bytes": Sb,
+                "us": round(ms * 1e3, 2), "algbw_gbs": round(alg, 2), "busbw_gbs": round(bus, 2),
+                "ctas_per_rank": info["ctas"], "blocks": sum(info["blocks_per_rank"]),
+                "instances": info["instances"], "linkmodel": info["linkmodel"], "fused": info["plan"]["fused"],
+                "sched": info.get("sched"), "err": err}
+    finally:
+        grp.destroy()
+
+
+def emit(d):
+    print(json.dumps(d), flush=True)
+
+
+which = sys.argv[1:] or ["c2"]
+if "c2" in which:
+    for coll in ("allreduce", "allgather"):
+        for dtype in ("bfloat16", "float32", "int32"):
+            sizes = [1 << k for k in range(10, 31, 2)] if dtype == "bfloat16" else [1 << 20, 64 << 20, 256 << 20]
+            for S in sizes:
+                emit(measure("ring", coll, "", BASE, S, dtype, iters=20 if S < (16 << 20) else 10))
+if "c3" in which:
+    for name, g in (("dbt", ""), ("hm", "g=4")):
+        for budget in (1, 2, 4, 8, 12, 16):
+            for S in (64 << 20, 256 << 20):
+                emit(measure(name, "allreduce", g, dict(chunkbytes=1 << 20, fifodepth=2, tbbudget=budget), S))
+    for S in (64 << 20, 256 << 20):
+        emit(measure("ring", "allreduce", "", dict(chunkbytes=1 << 20, fifodepth=2, instances=2), S))
+if "c4" in which:
+    for coll in ("allgather", "reducescatter"):
+        for fan in (2, 3):
+            for S in (4 << 20, 16 << 20, 64 << 20, 256 << 20):
+                emit(measure("synth", coll, f"seed=0 fanout={fan}", dict(instances=4, chunkbytes=1 << 20,
+                                                                          fifodepth=2), S))
+if "f2" in which:
+    for name, coll, g in (("hm", "allreduce", "g=4"), ("hm", "allgather", "g=4"), ("dbt", "allreduce", ""),
+                          ("synth", "allgather", "seed=0 fanout=2"), ("synth", "reducescatter", "seed=1 fanout=3")):
+        for sched in ("hpds", "rr"):
+            emit(measure(name, coll, g, dict(instances=4, chunkbytes=1 << 20, fifodepth=2, sched=sched),
+                         64 << 20))
