@@ -50,6 +50,7 @@ def parse():
     p.add_argument("--fifo-depth", type=int, default=0)
     p.add_argument("--nwarps", type=int, default=0)
     p.add_argument("--tma", type=int, default=-1, help="-1 = library default (on)")
+    p.add_argument("--direct", type=int, default=-1, help="direct push/pull transport (N=1 virtual ranks)")
     p.add_argument("--e2e-steps", type=int, default=3)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--sweep", default="", help="comma-separated MiB sizes for an extra busBW sweep")
@@ -215,9 +216,15 @@ def main():
     # default tuning: fill the SMs at N=1 (8 virtual ranks share one GPU)
     # default tuning (r01 sweeps, profiles/r01_*): 18 instances x 8 virtual ranks = 144 CTAs
     # (of 148 SMs), 4 MiB transfer chunks, FIFO depth 2 (FIFOs stay L2-resident)
+    # N=1: every virtual rank's buffers share one address space, so the direct transport
+    # (R23: push recv payloads, pull rrc operands; no FIFO staging) is the default there;
+    # multi-process (N>1) communicators use the staged FIFO transport.
     inst = args.instances or 18
-    opts = {"instances": inst, "chunkbytes": args.chunk_bytes or (4 << 20), "fifodepth": args.fifo_depth or 2,
-            "nwarps": args.nwarps or None, "tma": None if args.tma < 0 else args.tma}
+    direct = (0 if multi else 1) if args.direct < 0 else args.direct
+    opts = {"instances": inst, "chunkbytes": args.chunk_bytes or ((8 << 20) if direct else (4 << 20)),
+            "fifodepth": args.fifo_depth or 2,
+            "nwarps": args.nwarps or None, "tma": None if args.tma < 0 else args.tma,
+            "direct": direct}
     text = ir_text(R, args.algo, n, opts)
 
     if multi:
@@ -313,6 +320,8 @@ def main():
     if args.sweep:
         for mb in [float(x) for x in args.sweep.split(",") if x]:
             cnt = int(mb * (1 << 20)) // elt
+            if cnt > count:
+                continue  # sweep points are slices of the bench buffers
             s2 = {r: sends[r][:cnt] for r in my_ranks}
             r2 = {r: recvs[r][:cnt] for r in my_ranks}
             for _ in range(3):
@@ -353,7 +362,9 @@ def main():
         # => 9(N-1)/N * S.  Every byte crosses the L2 slices (LTS), whose throughput cap is
         # what also bounds the measured HBM copy peak, so that peak is the denominator.
         # dram_algorithmic = the user-buffer share 5(N-1)/N * S (FIFO slots stay in L2).
-        per_rank = 9.0 * (nr - 1) / nr * S
+        # direct transport (R23): no FIFO hop -- RS hop = pull-rrc reads s (peer) + s (own),
+        # writes s; AG hop = push-send reads s, writes s (peer) => 5(N-1)/N * S, all HBM.
+        per_rank = (5.0 if info.get("direct") else 9.0) * (nr - 1) / nr * S
         algo_bytes = per_rank * nr
         ach = algo_bytes / (ms * 1e-3) / 1e9
         roof = {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
@@ -384,7 +395,8 @@ def main():
                          f"{args.algo} allreduce, {n} GPUs (CUDA-IPC NVLink), {S >> 20} MiB per rank"),
             "nranks": n, "bytes_per_rank": S, "algo": args.algo, "instances": info["instances"],
             "chunkbytes": info["chunkbytes"], "fifodepth": info["fifodepth"], "nwarps": info["nwarps"],
-            "linkmodel": info["linkmodel"], "ctas_per_rank": info["ctas"], "blocks_total": sum(blocks),
+            "linkmodel": info["linkmodel"], "transport": "direct" if info.get("direct") else "staged-fifo",
+            "ctas_per_rank": info["ctas"], "blocks_total": sum(blocks),
             "sms_used": sms, "algbw_gbs": round(algbw, 2), "l2": "inputs > L2 on every rank (no flush)",
             "parallelism": "virtual-ranks" if not multi else f"ranks{n}",
         },

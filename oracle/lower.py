@@ -57,6 +57,10 @@ class Prim:
     cta: int = 0
     lane: str = "S"                   # S (send lane) | R (recv lane)
     deps: List[int] = field(default_factory=list)   # prim ids (same rank) waited on
+    ack_deps: List[int] = field(default_factory=list)  # direct: pull-sends completed by the peer's ack
+    direct: bool = False
+    pull: bool = False
+    rem_buf: Optional[str] = None     # direct: buffer of the peer location (push target / pull source)
     has_counter: bool = False
     pid: int = -1
 
@@ -65,6 +69,9 @@ class Prim:
         rt = tuple(tasks[self.recv_task]) if self.recv_task is not None else None
         st = tuple(tasks[self.send_task]) if self.send_task is not None else None
         return (self.kind, self.chunk, self.pc, rt, st, self.src_buf, self.dst_buf)
+
+
+DIRECT_KIND = {("send", False): "dsend", ("send", True): "psend", ("recv", False): "drecv", ("rrc", True): "prrc"}
 
 
 FUSED_KIND = {  # (recv op, store) -> fused name
@@ -87,6 +94,7 @@ class Plan:
     recv_groups: Dict[int, List[List[Tuple[int, str]]]]
     n_connections: Dict[int, int]
     fused: bool
+    direct: bool = False
 
     def ctas(self, r: int) -> int:
         return len(self.lanes[r])
@@ -132,7 +140,12 @@ def _greedy_merge(conns_act: Dict[Tuple[int, str], set]) -> List[List[Tuple[int,
     return groups
 
 
-def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None) -> Plan:
+def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool = False) -> Plan:
+    """``direct`` (reading R23): no FIFO staging; recv tasks are pushed into the
+    receiver's location after it posts "writable", rrc tasks are pulled from the
+    sender's location, whose completion is the receiver's read acknowledgement."""
+    if direct:
+        fuse = False
     edges, edge_rank = build_dag(ir)
     check_defined_reads(ir)
     if Pr is None:
@@ -170,6 +183,16 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None) -> Plan:
         rv = Prim(t.dst, t.op, t.chunk, pidx[i], recv_task=i, reduce=(t.op == RRC),
                   store=True, dst_buf=write_buf(coll, t.dst, t.chunk),
                   src_buf=read_buf(t.dst, t.chunk, t.step) if t.op == RRC else None)
+        if direct:
+            if t.op == RRC:
+                s.direct = s.pull = rv.direct = rv.pull = True
+                s.kind, rv.kind = "psend", "prrc"
+                rv.rem_buf = s.src_buf
+            else:
+                s.direct = rv.direct = True
+                s.kind, rv.kind = "dsend", "drecv"
+                s.rem_buf = rv.dst_buf
+                rv.store = False
         rv.pid = len(prims[t.dst]); prims[t.dst].append(rv); recv_of[i] = (t.dst, rv.pid)
 
     # -- connection activity + state-based merging (Eq. 7)
@@ -292,6 +315,12 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None) -> Plan:
                 r_l = sorted((p for p in final_list if p.lane == "R" and p.cta == c),
                              key=lambda p: p.pc)
                 lane_lists.append(([p.pid for p in s_l], [p.pid for p in r_l]))
+            # direct: dependencies on pull-sends complete with the receiver's ack and are
+            # never implied by lane order
+            if direct:
+                for p in final_list:
+                    p.ack_deps = [d for d in p.deps if final_list[d].kind == "psend"]
+                    p.deps = [d for d in p.deps if final_list[d].kind != "psend"]
             # drop dependencies implied by lane order
             pos_in_lane = {}
             for c, (sl, rl) in enumerate(lane_lists):
@@ -314,7 +343,7 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None) -> Plan:
     any_fused = bool(fuse) and any(absorbed[r] for r in range(N))
     plan = Plan(ir, model, edges, edge_rank, Pr, pidx, out_prims, lanes,
                 send_groups, recv_groups,
-                {r: len(act[r]) for r in range(N)}, any_fused)
+                {r: len(act[r]) for r in range(N)}, any_fused, direct)
     plan._act = act
     if fuse and any(absorbed[r] for r in range(N)):
         from .replay import deadlock_free

@@ -135,6 +135,10 @@ class Deadlock(RuntimeError):
 
 
 class _Sim:
+    """Processes = lanes x instances.  Per (link, instance): posted payload positions
+    (``fifo``) and a monotone ``credit``: the receiver's consumption (staged), its
+    "writable" posts (direct push) or its read acknowledgements (direct pull)."""
+
     def __init__(self, plan: Plan, n_mb: int, instances: int, K: int):
         self.plan, self.n_mb, self.I, self.K = plan, n_mb, instances, K
         self.tasks = plan.ir.transfers
@@ -149,54 +153,81 @@ class _Sim:
                 for lane, prog in (("S", sl), ("R", rl)):
                     if prog:
                         for inst in range(instances):
-                            self.procs.append([r, c, lane, inst, prog, 0, 0])
+                            self.procs.append([r, c, lane, inst, prog, 0, 0, 0])   # ..., k, j, phase
         self.done = defaultdict(int)
         self.fifo = defaultdict(dict)        # (link, inst) -> {pos: payload}
-        self.consumed = defaultdict(int)
+        self.credit = defaultdict(int)
         self.events = 0
 
     def _link(self, i):
         t = self.tasks[i]
         return (t.src, t.dst)
 
+    def pos(self, task, j):
+        return self.tpos[task] * self.n_mb + j
+
+    def deps_ok(self, r, p, j, inst) -> bool:
+        for d in p.deps:
+            if self.done[(r, d, inst)] < j + 1:
+                return False
+        for d in p.ack_deps:
+            t = self.plan.prims[r][d].send_task
+            if self.credit[(self._link(t), inst)] < self.pos(t, j) + 1:
+                return False
+        return True
+
     def enabled(self, pr) -> bool:
-        r, c, lane, inst, prog, k, j = pr
+        r, c, lane, inst, prog, k, j, phase = pr
         if k >= len(prog):
             return False
         p = self.plan.prims[r][prog[k]]
         if p.kind == "copy":
             return True
-        for d in p.deps:
-            if self.done[(r, d, inst)] < j + 1:
-                return False
-        if p.recv_task is not None:
-            pos = self.tpos[p.recv_task] * self.n_mb + j
-            if pos not in self.fifo[(self._link(p.recv_task), inst)]:
+        if p.kind == "drecv" and phase == 1:          # push receiver waiting for the payload
+            return self.pos(p.recv_task, j) in self.fifo[(self._link(p.recv_task), inst)]
+        if not self.deps_ok(r, p, j, inst):
+            return False
+        if p.recv_task is not None and p.kind != "drecv":
+            if self.pos(p.recv_task, j) not in self.fifo[(self._link(p.recv_task), inst)]:
                 return False
         if p.send_task is not None:
-            pos = self.tpos[p.send_task] * self.n_mb + j
-            if pos >= self.consumed[(self._link(p.send_task), inst)] + self.K:
-                return False
+            pos = self.pos(p.send_task, j)
+            cr = self.credit[(self._link(p.send_task), inst)]
+            if not p.direct:
+                if pos >= cr + self.K:
+                    return False
+            elif not p.pull:                          # push: receiver location writable
+                if cr < pos + 1:
+                    return False
         return True
 
     def finished(self) -> bool:
         return all(pr[5] >= len(pr[4]) for pr in self.procs)
 
     def fire(self, pr, action=None):
-        r, c, lane, inst, prog, k, j = pr
+        r, c, lane, inst, prog, k, j, phase = pr
         p = self.plan.prims[r][prog[k]]
+        if p.kind == "drecv" and phase == 0:          # post "writable", keep the micro-batch
+            key = (self._link(p.recv_task), inst)
+            self.credit[key] = max(self.credit[key], self.pos(p.recv_task, j) + 1)
+            pr[7] = 1
+            self.events += 1
+            return
+        pr[7] = 0
         incoming = None
         if p.recv_task is not None:
             key = (self._link(p.recv_task), inst)
-            pos = self.tpos[p.recv_task] * self.n_mb + j
+            pos = self.pos(p.recv_task, j)
             incoming = self.fifo[key].pop(pos)
-            assert pos == self.consumed[key], "out-of-order consumption"
-            self.consumed[key] += 1
+            if not p.direct:
+                assert pos == self.credit[key], "out-of-order consumption"
+                self.credit[key] += 1
+            elif p.pull:
+                self.credit[key] = max(self.credit[key], pos + 1)
         out = action(p, r, j, inst, incoming) if action else None
         if p.send_task is not None:
             key = (self._link(p.send_task), inst)
-            pos = self.tpos[p.send_task] * self.n_mb + j
-            self.fifo[key][pos] = out
+            self.fifo[key][self.pos(p.send_task, j)] = out
         if p.kind != "copy":
             self.done[(r, prog[k], inst)] = j + 1
         j += 1
@@ -235,7 +266,7 @@ class _Sim:
 
     def _stuck(self):
         out = []
-        for r, c, lane, inst, prog, k, j in self.procs:
+        for r, c, lane, inst, prog, k, j, _ in self.procs:
             if k < len(prog):
                 p = self.plan.prims[r][prog[k]]
                 out.append(f"rank{r} cta{c} {lane} inst{inst} at {p.kind} chunk{p.chunk} mb{j}")
@@ -310,6 +341,17 @@ def replay(plan: Plan, inputs: List[np.ndarray], dtype: str, count: int, op: str
                 bufs[r]["recv"][do + lo:do + hi] = bufs[r]["send"][so + lo:so + hi]
             return None
         lo, hi = g.slice(p.chunk, j, inst)
+        tasks = plan.ir.transfers
+        if p.kind == "dsend":                         # direct push: write the receiver's location
+            o = g.chunk_off(p.src_buf, p.chunk)
+            d, od = tasks[p.send_task].dst, g.chunk_off(p.rem_buf, p.chunk)
+            bufs[d][p.rem_buf][od + lo:od + hi] = bufs[r][p.src_buf][o + lo:o + hi]
+            return None
+        if p.kind in ("psend", "drecv"):              # flags only
+            return None
+        if p.kind == "prrc":                          # direct pull: read the sender's location
+            s_, os_ = tasks[p.recv_task].src, g.chunk_off(p.rem_buf, p.chunk)
+            incoming = bufs[s_][p.rem_buf][os_ + lo:os_ + hi].copy()
         if p.recv_task is None:                       # plain send
             o = g.chunk_off(p.src_buf, p.chunk)
             return bufs[r][p.src_buf][o + lo:o + hi].copy()
@@ -329,23 +371,26 @@ def replay(plan: Plan, inputs: List[np.ndarray], dtype: str, count: int, op: str
 
 # ------------------------------------------------------------------ I2 happens-before
 
-def happens_before_races(plan: Plan, n_mb: int = 2, instances: int = 1, K: int = 1):
+def happens_before_races(plan: Plan, n_mb: int = 2, instances: int = 1, K: int = 1, inplace: bool = False):
     """Return the list of conflicting, unordered access pairs (empty = I2 holds).
 
     Memory cells are (rank, buffer, chunk, micro-batch, instance) slices and FIFO
-    slots (link, instance, pos mod K).  Synchronisation edges: program order,
-    FIFO put -> take of a position, take of position p -> put of position p+K
-    (credit), and a primitive's micro-batch j -> waits on its counter for j."""
+    slots (link, instance, pos mod K).  Synchronisation edges: program order; a
+    payload/flag post of a position -> its consumer; a credit post of a position ->
+    the waiter it enables (staged: the sender of position p+K; direct push: the
+    sender of p; direct pull: dependents of the pull-send); a primitive's micro-batch j
+    -> waits on its counter for j."""
     sim = _Sim(plan, n_mb, instances, K)
     P = len(sim.procs)
     pid_of = {id(pr): k for k, pr in enumerate(sim.procs)}
     vc = [[0] * P for _ in range(P)]
-    put_vc, take_vc, done_vc = {}, {}, {}
+    put_vc, credit_vc, done_vc = {}, {}, {}
     cells = defaultdict(list)     # cell -> [(proc, own_clock, vc_snapshot, is_write)]
+    tasks = plan.ir.transfers
 
     def on_fire(pr, _):
         me = pid_of[id(pr)]
-        r, c, lane, inst, prog, k, j = pr
+        r, c, lane, inst, prog, k, j, phase = pr
         p = plan.prims[r][prog[k]]
         v = vc[me]
 
@@ -354,29 +399,52 @@ def happens_before_races(plan: Plan, n_mb: int = 2, instances: int = 1, K: int =
                 if o[q] > v[q]:
                     v[q] = o[q]
 
-        for d in p.deps:
-            join(done_vc[(r, d, inst, j)])
         acc = []
-        if p.recv_task is not None:
-            link = sim._link(p.recv_task)
-            pos = sim.tpos[p.recv_task] * n_mb + j
-            join(put_vc[(link, inst, pos)])
-            acc.append((("fifo", link, inst, pos % K), False))
-        if p.send_task is not None:
-            link = sim._link(p.send_task)
-            pos = sim.tpos[p.send_task] * n_mb + j
-            if pos - K >= 0:
-                join(take_vc[(link, inst, pos - K)])
-            acc.append((("fifo", link, inst, pos % K), True))
+        rlink = sim._link(p.recv_task) if p.recv_task is not None else None
+        slink = sim._link(p.send_task) if p.send_task is not None else None
+        rpos = sim.pos(p.recv_task, j) if p.recv_task is not None else None
+        spos = sim.pos(p.send_task, j) if p.send_task is not None else None
+        if p.kind == "drecv" and phase == 1:
+            join(put_vc[(rlink, inst, rpos)])
+        elif p.kind != "copy":
+            for d in p.deps:
+                join(done_vc[(r, d, inst, j)])
+            for d in p.ack_deps:
+                t = plan.prims[r][d].send_task
+                join(credit_vc[(sim._link(t), inst, sim.pos(t, j))])
+            if p.recv_task is not None and p.kind != "drecv":
+                join(put_vc[(rlink, inst, rpos)])
+            if p.send_task is not None:
+                if not p.direct:
+                    if spos - K >= 0:
+                        join(credit_vc[(slink, inst, spos - K)])
+                elif not p.pull:
+                    join(credit_vc[(slink, inst, spos)])
         jj = 0 if p.kind == "copy" else j
         if p.kind == "copy":
             acc.append(((r, "send", p.chunk, -1, -1), False))
             acc.append(((r, "recv", p.chunk, -1, -1), True))
-        else:
+        elif p.kind == "dsend":
+            acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
+            acc.append(((tasks[p.send_task].dst, p.rem_buf, p.chunk, jj, inst), True))
+        elif p.kind == "prrc":
+            acc.append(((tasks[p.recv_task].src, p.rem_buf, p.chunk, jj, inst), False))
+            acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
+            acc.append(((r, p.dst_buf, p.chunk, jj, inst), True))
+        elif p.kind not in ("psend", "drecv"):
+            if p.recv_task is not None:
+                acc.append((("fifo", rlink, inst, rpos % K), False))
+            if p.send_task is not None:
+                acc.append((("fifo", slink, inst, spos % K), True))
             if p.src_buf and (p.recv_task is None or p.reduce):
                 acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
             if p.recv_task is not None and p.store:
                 acc.append(((r, p.dst_buf, p.chunk, jj, inst), True))
+        if inplace and p.kind == "copy":
+            acc = []  # in-place, the output already holds the input: the copy does nothing
+        if inplace:  # in-place: a location's send- and receive-buffer copies are one memory
+            acc = [((cl[0], "recv" if cl[1] == "send" else cl[1]) + cl[2:], w) if cl[0] != "fifo" else (cl, w)
+                   for cl, w in acc]
         v[me] += 1
         snap = list(v)
         for cell, w in acc:
@@ -386,14 +454,13 @@ def happens_before_races(plan: Plan, n_mb: int = 2, instances: int = 1, K: int =
                 for jx in range(n_mb):
                     for ix in range(instances):
                         cells[(cell[0], cell[1], cell[2], jx, ix)].append((me, v[me], snap, w))
-        if p.recv_task is not None:
-            link = sim._link(p.recv_task)
-            pos = sim.tpos[p.recv_task] * n_mb + j
-            take_vc[(link, inst, pos)] = snap
+        if p.kind == "drecv" and phase == 0:
+            credit_vc[(rlink, inst, rpos)] = snap          # "writable"
+            return
+        if p.recv_task is not None and p.kind != "drecv":
+            credit_vc[(rlink, inst, rpos)] = snap          # consumed / read acknowledged
         if p.send_task is not None:
-            link = sim._link(p.send_task)
-            pos = sim.tpos[p.send_task] * n_mb + j
-            put_vc[(link, inst, pos)] = snap
+            put_vc[(slink, inst, spos)] = snap             # payload / "written" / "readable"
         if p.kind != "copy":
             done_vc[(r, prog[k], inst, j)] = snap
 

@@ -131,7 +131,9 @@ struct Options {
   int tma_stages = 4;
   int trace = 0;
   int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
+  int direct = 0;    // direct transport (R23): virtual ranks / single-process only
   int l2hint = 1;
+  int tma_min = 32768;
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
 };
 
@@ -172,6 +174,8 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "trace") o.trace = (int)to_long(v, k);
   else if (k == "l2hint") o.l2hint = (int)to_long(v, k);
   else if (k == "prefetch") o.prefetch = (int)to_long(v, k);
+  else if (k == "tmamin") o.tma_min = (int)to_long(v, k);
+  else if (k == "direct") o.direct = (int)to_long(v, k);
   else if (k == "sched") {
     if (v == "hpds") o.sched = 0;
     else if (v == "rr") o.sched = 1;
@@ -192,7 +196,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -213,9 +217,9 @@ Plan lower_with(const Ir& ir, LinkModel m, const Options& o) {
   if (o.sched == 1) {
     Dag d = build_dag(ir);
     auto pr = round_robin(ir, d, m);
-    return lower(ir, m, o.fuse, &pr);
+    return lower(ir, m, o.fuse, &pr, o.direct != 0);
   }
-  return lower(ir, m, o.fuse);
+  return lower(ir, m, o.fuse, nullptr, o.direct != 0);
 }
 
 Plan make_plan(const Ir& ir, Options& o) {
@@ -414,7 +418,7 @@ std::string info_json(const AlgoShared& a) {
   o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
     << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"tma\":" << a.opt.tma
     << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"l2hint\":" << a.opt.l2hint << ",\"prefetch\":" << a.opt.prefetch << ",\"sched\":\""
-    << (a.opt.sched ? "rr" : "hpds") << "\"" << ",\"linkmodel\":\""
+    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"linkmodel\":\""
     << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
     << ",\"ctas\":[";
   for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];
@@ -440,6 +444,7 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.trace = a.opt.trace;
   co.l2hint = a.opt.l2hint;
   co.prefetch = a.opt.prefetch;
+  co.tma_min = a.opt.tma_min;
   std::string src = codegen(a.plan, a.lay, co);
   if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
     if (FILE* f = fopen((std::string(dump) + "_" + a.ir.name + "_" + coll_name(a.ir.coll) + ".cu").c_str(), "w")) {
@@ -697,6 +702,9 @@ rescclAlgo* load_algo(rescclComm* comm, const std::string& text) {
     }
   } else {
     s = build_algo(text, comm->nranks);
+    if (s->opt.direct)
+      fail(rescclInvalidUsage, "direct=1 needs every rank's buffers in one address space (virtual ranks); "
+                               "multi-process communicators use the staged FIFO transport");
     size_t need = (size_t)s->lay.region_bytes;
     if (comm->arena_used + need > comm->arena_bytes)
       fail(rescclInvalidUsage, "FIFO arena exhausted: need " + std::to_string(comm->arena_used + need) +
@@ -1121,6 +1129,7 @@ rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo
   co.trace = o.trace;
   co.l2hint = o.l2hint;
   co.prefetch = o.prefetch;
+  co.tma_min = o.tma_min;
   write_out(codegen(p, L, co), src, len);
   API_END
 }
@@ -1141,6 +1150,7 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
   co.trace = o.trace;
   co.l2hint = o.l2hint;
   co.prefetch = o.prefetch;
+  co.tma_min = o.tma_min;
   co.gpu_scope = true;
   auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, true);
   if (cubin_bytes) *cubin_bytes = cub.size();

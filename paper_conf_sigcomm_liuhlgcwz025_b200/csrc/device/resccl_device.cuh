@@ -58,7 +58,7 @@ struct KArgs {
   u64* trace;                         // RESCCL_TRACE: 4 x u64 per (block, lane), host-mapped
 };
 
-enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16 };
+enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16, kDirect = 32, kPull = 64 };
 enum : int { BufSend = 0, BufRecv = 1, BufScratch = 2 };
 enum : int { CollAllGather = 0, CollReduceScatter = 1, CollAllReduce = 2 };
 enum : int { OpSum = 0, OpMax = 1, OpMin = 2 };
@@ -454,7 +454,13 @@ struct PrimDesc {
   i64 in_data, in_flag, in_cred, in_pos, in_n;
   i64 out_data, out_flag, out_cred, out_pos, out_n;
   i64 ctr;
+  int rem_rank, rem_buf;       // direct mode: the peer location (push target / pull source)
+  // dependency k is satisfied for micro-batch j when the u64 at deps[k] in this rank's
+  // region reaches dep_n[k] * mb_base + dep_pos[k] * n_mb + j + 1: a completion counter
+  // (n = 1, pos = 0) or, for a direct pull-send, the receiver's read credit of its link.
   i64 deps[RESCCL_MAXDEPS];
+  i64 dep_n[RESCCL_MAXDEPS];
+  i64 dep_pos[RESCCL_MAXDEPS];
 };
 
 // Layout constants shared by every primitive of a plan (emitted by the generator):
@@ -469,8 +475,13 @@ struct PrimPtrs {
   u64* out_flag;
   u64* out_cred;     // credit counter the receiver writes back (own arena)
   u64* ctr;
+  const char* R;     // direct mode: peer location base (chunk start)
   i64 len;           // chunk length (elements)
 };
+
+__device__ __forceinline__ u64 dep_target(const KArgs& a, const PrimDesc& d, int k, int j) {
+  return (u64)d.dep_n[k] * a.mb_base + (u64)d.dep_pos[k] * a.n_mb + j + 1;
+}
 
 __device__ __forceinline__ void slice_of(const KArgs& a, i64 len, int j, int inst, i64& lo, i64& hi) {
   lo = (i64)j * a.M + (i64)inst * a.Mi;
@@ -497,14 +508,18 @@ __device__ __forceinline__ bool mb_ready(const Lane& L, const PrimDesc& d, const
   const KArgs& a = *L.a;
   const u64 mb_base = a.mb_base;
   for (int k = 0; k < d.ndeps; ++k)
-    if (ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) < mb_base + j + 1) return false;
+    if (ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) < dep_target(a, d, k, j)) return false;
   if (F & kRecv) {
     const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
     if (ld_acquire(p.in_flag + (in_seq % RESCCL_K)) < in_seq + 1) return false;
   }
   if (F & kSend) {
     const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
-    if (out_seq + 1 > (u64)RESCCL_K && ld_acquire(p.out_cred) < out_seq + 1 - RESCCL_K) return false;
+    if (F & kDirect) {  // push: the receiver's location must be writable
+      if (ld_acquire(p.out_cred) < out_seq + 1) return false;
+    } else if (out_seq + 1 > (u64)RESCCL_K && ld_acquire(p.out_cred) < out_seq + 1 - RESCCL_K) {
+      return false;
+    }
   }
   return true;
 }
@@ -521,9 +536,14 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
     if (L.tid == 0) {
       bool ok = true;
       for (int k = 0; k < d.ndeps && ok; ++k)
-        ok = L.wait_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), mb_base + j + 1);
+        ok = L.wait_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, j));
       if (ok && (F & kRecv)) ok = L.wait_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1);
-      if (ok && (F & kSend) && out_seq + 1 > (u64)RESCCL_K) ok = L.wait_ge(p.out_cred, out_seq + 1 - RESCCL_K);
+      if (ok && (F & kSend)) {
+        if (F & kDirect)
+          ok = L.wait_ge(p.out_cred, out_seq + 1);
+        else if (out_seq + 1 > (u64)RESCCL_K)
+          ok = L.wait_ge(p.out_cred, out_seq + 1 - RESCCL_K);
+      }
       if (!ok) *L.abort_flag = 1;
     }
     L.sync();
@@ -532,9 +552,11 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
     slice_of(a, p.len, j, L.inst, lo, hi);
     const char* Aj = p.A ? p.A + lo * T::kSize : nullptr;
     char* D1j = p.D1 ? p.D1 + lo * T::kSize : nullptr;
-    const char* Bj = (F & kRecv) ? p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
-    char* D2j = (F & kSend) ? p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT : nullptr;
-    move<T, OP, F, 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
+    const char* Bj = (F & kRecv) ? ((F & kDirect) ? p.R + lo * T::kSize : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT)
+                                 : nullptr;
+    char* D2j = (F & kSend) ? ((F & kDirect) ? (char*)p.R + lo * T::kSize : p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT)
+                            : nullptr;
+    move<T, OP, F & ~(kDirect | kPull), 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
     L.sync();
     if (L.tid == 0) post_mb<F>(a, d, p, j);
   }
@@ -626,10 +648,11 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
       if (F & kReduce) {
         const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + lj;
+        const char* bsrc = (F & kDirect) ? p.R + lo_l * T::kSize + off
+                                         : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off;
         mbar_expect_tx(L.full + 8 * s, 2 * nb);
         tma_load(sa, p.A + lo_l * T::kSize + off, nb, L.full + 8 * s, pol_first);
-        tma_load(sa + (u32)RESCCL_TMA_TILE, p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off, nb,
-                 L.full + 8 * s, pol_first);
+        tma_load(sa + (u32)RESCCL_TMA_TILE, bsrc, nb, L.full + 8 * s, pol_first);
       } else {
         const char* src;
         if (F & kRecv) {
@@ -663,8 +686,12 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
       if (F & kStore) tma_store(p.D1 + lo_s * T::kSize + off, sa, nb, pol_first);
       if (F & kSend) {
-        const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + sj;
-        tma_store(p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + off, sa, nb, pol_last);
+        if (F & kDirect) {
+          tma_store((char*)p.R + lo_s * T::kSize + off, sa, nb, pol_first);
+        } else {
+          const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + sj;
+          tma_store(p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + off, sa, nb, pol_last);
+        }
       }
       tma_commit();
       if (F & kReduce) L.comp_use[s]++;
@@ -682,10 +709,15 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       if (e0 < hi_h) {
         const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + pj;
         const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + pj;
-        const char* Bj = (F & kRecv) ? p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + nb_p : nullptr;
-        char* D2j = (F & kSend) ? p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + nb_p : nullptr;
+        const char* Bj = (F & kRecv) ? ((F & kDirect) ? p.R + e0 * T::kSize
+                                                     : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
+                                     : nullptr;
+        char* D2j = (F & kSend) ? ((F & kDirect) ? (char*)p.R + e0 * T::kSize
+                                                 : p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
+                                : nullptr;
         for (i64 e = 0; e < hi_h - e0; ++e)
-          elem_move<T, OP>(F, p.A ? p.A + e0 * T::kSize : nullptr, Bj, p.D1 ? p.D1 + e0 * T::kSize : nullptr, D2j, e);
+          elem_move<T, OP>(F & ~(kDirect | kPull), p.A ? p.A + e0 * T::kSize : nullptr, Bj,
+                           p.D1 ? p.D1 + e0 * T::kSize : nullptr, D2j, e);
       }
       fence_proxy_async();
       post_mb<F>(a, d, p, pj);
@@ -761,6 +793,74 @@ __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const Prim
   return true;
 }
 
+// Direct-mode primitives that move no data (leader only): a pull-send posts "readable"
+// for each micro-batch once its dependencies hold; a push-receive posts "writable"
+// (credit) as soon as its dependencies hold -- running ahead of the payloads -- and
+// completes a micro-batch when the sender's "written" flag arrives.
+template <int F>
+__device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
+  const KArgs& a = *L.a;
+  const int nmb = a.n_mb;
+  const u64 mb_base = a.mb_base;
+  int wp = 0, dj = 0;  // push-receive: writable posted / completed micro-batches
+  u64 t_idle = 0;
+  u32 spins = 0;
+  while ((F & kSend) ? wp < nmb : dj < nmb) {
+    bool prog = false;
+    if (wp < nmb) {
+      bool ok = true;
+      for (int k = 0; k < d.ndeps && ok; ++k)
+        ok = ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) >= dep_target(a, d, k, wp);
+      if (ok) {
+        fence_release();
+        if (F & kSend) {
+          const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + wp;
+          st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);
+        } else {
+          const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + wp;
+          st_relaxed(p.in_cred, in_seq + 1);
+        }
+        ++wp;
+        prog = true;
+      }
+    }
+    if (!(F & kSend) && dj < wp) {
+      const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + dj;
+      if (ld_acquire(p.in_flag + (in_seq % RESCCL_K)) >= in_seq + 1) {
+        fence_release();
+        if (d.ctr >= 0) st_relaxed(p.ctr, mb_base + dj + 1);
+        ++dj;
+        prog = true;
+      }
+    }
+    if (prog) {
+#if RESCCL_TRACE
+      if (t_idle) L.wait_ns += globaltimer() - t_idle;
+#endif
+      spins = 0;
+      t_idle = 0;
+    } else {
+#if RESCCL_TRACE
+      if (t_idle == 0) t_idle = globaltimer();
+#endif
+      if (++spins > 32) nanosleep_(20);
+      if ((spins & 255) == 0) {
+        const u64 now = globaltimer();
+        if (t_idle == 0) t_idle = now;
+        else if (now - t_idle > a.timeout_ns) {
+          atomicCAS(a.err, 0, kErrTimeout);
+          *L.abort_flag = 1;
+          return false;
+        }
+      }
+    }
+  }
+#if RESCCL_TRACE
+  if (t_idle) L.wait_ns += globaltimer() - t_idle;
+#endif
+  return true;
+}
+
 template <class T, int OP, int F>
 __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
   const KArgs& a = *L.a;
@@ -790,9 +890,17 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
   p.out_flag = (F & kSend) ? at(peer, d.out_flag + (i64)L.inst * RESCCL_FLAGSTRIDE) : nullptr;
   p.out_cred = at(L.self, d.out_cred + (i64)L.inst * 128);
   p.ctr = at(L.self, d.ctr + (i64)L.inst * 128);
+  p.R = (F & kDirect) ? buf_ptr(a, d.rem_rank, d.rem_buf) + chunk_off<RESCCL_COLL>(d.rem_buf, c, a.C) * T::kSize
+                      : nullptr;
+  if ((F & kDirect) && (((F & kSend) && (F & kPull)) || ((F & kRecv) && !(F & kPull))))
+    return L.tid == 0 ? run_flags<F>(L, d, p) : true;
+#ifndef RESCCL_TMA_MIN
+#define RESCCL_TMA_MIN 32768
+#endif
 #if RESCCL_TMA
-  const unsigned long long al = (unsigned long long)p.A | (unsigned long long)p.D1;
-  if ((al & 15) == 0) {
+  // small slices are latency-bound: the register path saves two bulk-copy round trips
+  const unsigned long long al = (unsigned long long)p.A | (unsigned long long)p.D1 | (unsigned long long)p.R;
+  if ((al & 15) == 0 && a.Mi * T::kSize >= RESCCL_TMA_MIN) {
     if (L.tid == 0) return pipe_leader<T, OP, F>(L, d, p);
     if (L.tid < 32) return true;
     if (F & kReduce) return pipe_compute<T, OP, F>(L, d, p, L.tid - 32, L.nthreads - 32);

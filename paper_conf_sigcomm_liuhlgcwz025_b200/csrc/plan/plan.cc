@@ -12,6 +12,10 @@ namespace resccl {
 
 const char* Prim::kind_name() const {
   if (flags & kCopy) return "copy";
+  if (flags & kDirect) {
+    if (flags & kSend) return (flags & kPull) ? "psend" : "dsend";
+    return (flags & kPull) ? "prrc" : "drecv";
+  }
   bool rv = flags & kRecv, sd = flags & kSend, red = flags & kReduce, st = flags & kStore;
   if (!rv) return "send";
   if (!sd) return red ? "rrc" : "recv";
@@ -343,6 +347,20 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
         std::stable_sort(l.begin(), l.end(), [&](int a, int b) { return fin[a].pc < fin[b].pc; });
         (lane == 0 ? RP.ctas[c].first : RP.ctas[c].second) = l;
       }
+    // direct mode: a dependency on a pull-send completes with the receiver's ack; it
+    // is never implied by lane order (the pull-send itself returns before the read)
+    if (P.direct) {
+      for (auto& p : fin) {
+        std::vector<int> keep;
+        for (int d : p.deps) {
+          if ((fin[d].flags & kDirect) && (fin[d].flags & kSend) && (fin[d].flags & kPull))
+            p.ack_deps.push_back(d);
+          else
+            keep.push_back(d);
+        }
+        p.deps = keep;
+      }
+    }
     // drop dependencies implied by lane order
     std::map<int, std::tuple<int, int, int>> where;
     for (int c = 0; c < ncta; ++c) {
@@ -366,10 +384,12 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
   }
 }
 
-Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<int>>* pr_in) {
+Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<int>>* pr_in, bool direct) {
   Plan P;
   P.ir = ir;
   P.model = m;
+  P.direct = direct;
+  if (direct) fuse = false;
   P.dag = build_dag(ir);
   P.pr = pr_in ? *pr_in : hpds(ir, P.dag, m);
   const int T = (int)ir.t.size(), N = ir.nranks;
@@ -432,6 +452,18 @@ Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<i
     rv.dst_buf = write_buf(ir.coll, x.dst, x.chunk);
     rv.src_buf = x.op == Op::Rrc ? read_buf(x.dst, x.chunk, x.step) : BufNone;
     rv.lane = 1;
+    if (direct) {
+      if (x.op == Op::Rrc) {  // pull: receiver reads the sender's location
+        s.flags |= kDirect | kPull;
+        rv.flags |= kDirect | kPull;
+        rv.rem_buf = s.src_buf;
+      } else {                // push: sender writes the receiver's location
+        s.flags |= kDirect;
+        s.rem_buf = rv.dst_buf;
+        rv.flags = kRecv | kDirect;
+      }
+      raw[x.src].prims[send_of[i].second] = s;
+    }
     recv_of[i] = {x.dst, (int)raw[x.dst].prims.size()};
     raw[x.dst].prims.push_back(rv);
   }
@@ -516,12 +548,18 @@ Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<i
 }
 
 // ----------------------------------------------------------------------------- I4 simulation
+// Blocking semantics per (primitive, micro-batch) of a lane; per link a set of posted
+// payload positions ("flags") and a monotone credit counter.  Staged: the receiver's
+// consumption is the credit; a sender may run K positions ahead.  Direct (R23): a push
+// receiver first posts "writable" (credit) once its dependencies hold, then waits for the
+// payload; a push sender waits for that credit; a pull sender only posts "readable" and
+// its completion (for dependents) is the receiver's read credit.
 bool deadlock_free(const Plan& P, int K, int n_mb, std::string* why) {
   const Ir& ir = P.ir;
   struct Proc {
     int r, cta, lane;
     const std::vector<int>* prog;
-    int k = 0, j = 0;
+    int k = 0, j = 0, phase = 0;
   };
   std::vector<Proc> procs;
   for (int r = 0; r < ir.nranks; ++r)
@@ -533,33 +571,59 @@ bool deadlock_free(const Plan& P, int K, int n_mb, std::string* why) {
     }
   std::map<std::pair<int, int>, int> done;  // (rank, prim) -> #micro-batches finished
   std::map<std::pair<int, int>, std::set<long>> produced;
-  std::map<std::pair<int, int>, long> consumed;
+  std::map<std::pair<int, int>, long> credit;
   auto link = [&](int t) { return std::make_pair(ir.t[t].src, ir.t[t].dst); };
+  auto pos_of = [&](int t, int j) { return (long)P.link_pos[t] * n_mb + j; };
+  auto deps_ok = [&](const Proc& p, const Prim& pm) {
+    for (int d : pm.deps)
+      if (done[{p.r, d}] < p.j + 1) return false;
+    for (int d : pm.ack_deps) {
+      int t = P.ranks[p.r].prims[d].send_task;
+      if (credit[link(t)] < pos_of(t, p.j) + 1) return false;
+    }
+    return true;
+  };
   auto enabled = [&](Proc& p) {
     if (p.k >= (int)p.prog->size()) return false;
     const Prim& pm = P.ranks[p.r].prims[(*p.prog)[p.k]];
     if (pm.flags & kCopy) return true;
-    for (int d : pm.deps)
-      if (done[{p.r, d}] < p.j + 1) return false;
-    if (pm.recv_task >= 0) {
-      long pos = (long)P.link_pos[pm.recv_task] * n_mb + p.j;
-      if (!produced[link(pm.recv_task)].count(pos)) return false;
+    const bool direct = pm.flags & kDirect, pull = pm.flags & kPull;
+    if (direct && (pm.flags & kRecv) && !pull && p.phase == 1)  // push receiver waiting for payload
+      return produced[link(pm.recv_task)].count(pos_of(pm.recv_task, p.j)) > 0;
+    if (!deps_ok(p, pm)) return false;
+    if (pm.flags & kRecv) {
+      if (!direct || pull)
+        if (!produced[link(pm.recv_task)].count(pos_of(pm.recv_task, p.j))) return false;
     }
-    if (pm.send_task >= 0) {
-      long pos = (long)P.link_pos[pm.send_task] * n_mb + p.j;
-      if (pos >= consumed[link(pm.send_task)] + K) return false;
+    if (pm.flags & kSend) {
+      long pos = pos_of(pm.send_task, p.j);
+      if (!direct) {
+        if (pos >= credit[link(pm.send_task)] + K) return false;
+      } else if (!pull) {
+        if (credit[link(pm.send_task)] < pos + 1) return false;
+      }
     }
     return true;
   };
   auto fire = [&](Proc& p) {
     int pid = (*p.prog)[p.k];
     const Prim& pm = P.ranks[p.r].prims[pid];
-    if (pm.recv_task >= 0) {
-      long pos = (long)P.link_pos[pm.recv_task] * n_mb + p.j;
-      produced[link(pm.recv_task)].erase(pos);
-      consumed[link(pm.recv_task)] += 1;
+    const bool direct = pm.flags & kDirect, pull = pm.flags & kPull;
+    if (direct && (pm.flags & kRecv) && !pull && p.phase == 0) {  // post "writable", keep the micro-batch
+      credit[link(pm.recv_task)] = std::max(credit[link(pm.recv_task)], pos_of(pm.recv_task, p.j) + 1);
+      p.phase = 1;
+      return;
     }
-    if (pm.send_task >= 0) produced[link(pm.send_task)].insert((long)P.link_pos[pm.send_task] * n_mb + p.j);
+    p.phase = 0;
+    if (pm.recv_task >= 0) {
+      long pos = pos_of(pm.recv_task, p.j);
+      if (!direct || pull) produced[link(pm.recv_task)].erase(pos);
+      if (!direct)
+        credit[link(pm.recv_task)] += 1;
+      else if (pull)
+        credit[link(pm.recv_task)] = std::max(credit[link(pm.recv_task)], pos + 1);
+    }
+    if (pm.send_task >= 0) produced[link(pm.send_task)].insert(pos_of(pm.send_task, p.j));
     if (!(pm.flags & kCopy)) done[{p.r, pid}] = p.j + 1;
     p.j++;
     if (p.j >= ((pm.flags & kCopy) ? 1 : n_mb)) {
@@ -610,7 +674,7 @@ std::string plan_json(const Plan& P) {
   const Ir& ir = P.ir;
   o << "{\"name\":\"" << ir.name << "\",\"coll\":\"" << coll_name(ir.coll) << "\",\"nranks\":" << ir.nranks
     << ",\"model\":\"" << (P.model == LinkModel::Pair ? "pair" : "port") << "\",\"fused\":"
-    << (P.fused ? "true" : "false") << ",\"n_edges\":" << P.dag.edges.size() << ",\"tasks\":[";
+    << (P.fused ? "true" : "false") << ",\"direct\":" << (P.direct ? "true" : "false") << ",\"n_edges\":" << P.dag.edges.size() << ",\"tasks\":[";
   for (size_t i = 0; i < ir.t.size(); ++i) {
     auto& x = ir.t[i];
     o << (i ? "," : "") << "[" << x.src << "," << x.dst << "," << x.step << "," << x.chunk << ",\""
@@ -652,8 +716,11 @@ std::string plan_json(const Plan& P) {
       o << (k ? "," : "") << "{\"kind\":\"" << p.kind_name() << "\",\"chunk\":" << p.chunk << ",\"pc\":" << p.pc
         << ",\"recv_task\":" << p.recv_task << ",\"send_task\":" << p.send_task << ",\"src\":\""
         << buf_name(p.src_buf) << "\",\"dst\":\"" << buf_name(p.dst_buf) << "\",\"cta\":" << p.cta
-        << ",\"lane\":" << p.lane << ",\"counter\":" << (p.has_counter ? "true" : "false") << ",\"deps\":[";
+        << ",\"lane\":" << p.lane << ",\"counter\":" << (p.has_counter ? "true" : "false")
+        << ",\"rem\":\"" << buf_name(p.rem_buf) << "\",\"deps\":[";
       for (size_t d = 0; d < p.deps.size(); ++d) o << (d ? "," : "") << p.deps[d];
+      o << "],\"ack_deps\":[";
+      for (size_t d = 0; d < p.ack_deps.size(); ++d) o << (d ? "," : "") << p.ack_deps[d];
       o << "]}";
     }
     o << "]}";

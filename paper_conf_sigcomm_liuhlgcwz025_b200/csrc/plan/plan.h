@@ -43,6 +43,12 @@ enum PrimFlags : int {
   kReduce = 4,   // value = local (+) incoming
   kStore = 8,    // stores the value locally
   kCopy = 16,    // local copy send buffer -> receive buffer
+  // direct transport (reading R23): no FIFO staging.  recv tasks are pushed by the
+  // sender straight into the receiver's location once the receiver posted "writable";
+  // rrc tasks are pulled: the sender only posts "readable" and the receiver reads the
+  // sender's location; the sender's completion is the receiver's read acknowledgement.
+  kDirect = 32,
+  kPull = 64,    // with kDirect: payload read from the peer's buffer (rrc tasks)
 };
 
 struct Prim {
@@ -56,6 +62,8 @@ struct Prim {
   int cta = 0;
   int lane = 0;         // 0 = send lane, 1 = recv lane
   std::vector<int> deps;  // prim ids on this rank whose same-micro-batch completion is awaited
+  std::vector<int> ack_deps;  // direct mode: pull-send prims whose completion is the peer's ack
+  int rem_buf = BufNone;  // direct mode: buffer of the peer's location (push target / pull source)
   bool has_counter = false;
   const char* kind_name() const;
 };
@@ -84,12 +92,14 @@ struct Plan {
   std::vector<int> pidx;             // task -> pipeline index
   std::vector<RankPlan> ranks;
   bool fused = false;
+  bool direct = false;
   // FIFO order of every link: tasks sorted by pipeline index
   std::vector<int> link_pos;  // task -> position on its link
   std::vector<int> link_len;  // task -> #tasks on its link
 };
 
-Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<int>>* pr = nullptr);
+Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<int>>* pr = nullptr,
+           bool direct = false);
 
 // Control-only blocking simulation of the lowered plan (I4).  Returns true if every
 // lane completes for FIFO depth K and n_mb micro-batches.

@@ -28,7 +28,8 @@ def _positions(geo, c, rng, n_rand=3000):
 
 @pytest.mark.timeout(600)
 @pytest.mark.parametrize("algo,n,size_mb,dtype,opts", [
-    ("ring", 8, 256, "bfloat16", dict(instances=16, chunkbytes=2 << 20, fifodepth=2)),   # bench.py default
+    ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=4 << 20, fifodepth=2)),   # bench.py default
+    ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=4 << 20, fifodepth=2, direct=1)),
     ("ring", 8, 64, "float32", dict(instances=16, chunkbytes=2 << 20, fifodepth=2)),
     ("hm", 8, 64, "bfloat16", dict(instances=4, chunkbytes=1 << 20, fifodepth=2)),
     ("dbt", 8, 64, "float16", dict(instances=4, chunkbytes=1 << 20, fifodepth=2)),

@@ -203,3 +203,31 @@ def test_load_rejects_bad_ir():
             grp.comms[0].load("algo name=x coll=allreduce nranks=2 nchunks=2\nt 0 1 0 0 rrc\nt 1 0 0 0 rrc\n")
     finally:
         grp.destroy()
+
+
+@pytest.mark.parametrize("name,coll,n,kw", ALGOS)
+@pytest.mark.parametrize("dtype", ["bfloat16", "int32"])
+def test_direct_transport_bit_exact(name, coll, n, kw, dtype):
+    """Direct push/pull transport (R23) on virtual ranks: same bytes as the oracle."""
+    g = oir.generate(name, coll, n, **kw)
+    count = 3 * 4096 + 77
+    text = _hdr(g, chunkbytes=4096, instances=2, direct=1)
+    xs = _inputs(coll, dtype, n, count)
+    outs, info, err = run_virtual(R, text, coll, xs, dtype, count)
+    assert err == 0 and info["direct"] == 1
+    exp = oracle_expect(g, xs, dtype, count, chunk_bytes=4096, instances=2, K=2)
+    _check_bytes(outs, exp, coll, n, count)
+
+
+@pytest.mark.parametrize("coll", ["allreduce", "allgather", "reducescatter"])
+@pytest.mark.parametrize("count", [1, 129, 4097, 300001])
+def test_direct_edge_counts_inplace(coll, count):
+    n = 8
+    g = oir.generate("ring", coll, n)
+    xs = _inputs(coll, "bfloat16", n, count, seed=4)
+    for inplace in (False, True):
+        outs, _, err = run_virtual(R, _hdr(g, chunkbytes=65536, instances=3, direct=1), coll, xs, "bfloat16",
+                                   count, inplace=inplace)
+        assert err == 0
+        exp = oracle_expect(g, xs, "bfloat16", count, chunk_bytes=65536, instances=3)
+        _check_bytes(outs, exp, coll, n, count)

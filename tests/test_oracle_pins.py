@@ -420,7 +420,8 @@ def test_happens_before_no_races(name, coll, n, model):
     """I2 (proof): every conflicting access pair is ordered by happens-before."""
     pl = lower.lower(_gen(name, coll, n), model)
     for n_mb, K in ((1, 1), (2, 1), (3, 2)):
-        assert replay.happens_before_races(pl, n_mb=n_mb, instances=1, K=K) == []
+        for inplace in (False, True):
+            assert replay.happens_before_races(pl, n_mb=n_mb, instances=1, K=K, inplace=inplace) == []
 
 
 def test_exhaustive_interleavings_tiny():
@@ -526,3 +527,45 @@ def test_invalid_ir_rejected():
 def test_text_roundtrip():
     for g in (ir.hm_allreduce(2, 4), ir.synth_reducescatter(8, 3, 2)):
         assert ir.parse_text(g.to_text()) == g
+
+
+# ----------------------------------------------------------------------------- direct transport (R23)
+
+@pytest.mark.parametrize("name,coll,n", ALGOS)
+def test_direct_transport_replay_and_races(name, coll, n):
+    """Direct push/pull semantics give the definition (int32), the staged mode's bytes
+    (fp32), no happens-before races and no deadlock."""
+    g = _gen(name, coll, n)
+    pd = lower.lower(g, "pair", direct=True)
+    ps = lower.lower(g, "pair")
+    cnt = 500
+    m = cnt * n if coll == "reducescatter" else cnt
+    xs = inp.all_inputs("int32", 4, n, m)
+    out = replay.replay(pd, xs, "int32", cnt, chunk_bytes=256, instances=2, K=1)
+    for a, b in zip(out, _defn(coll, xs, "int32")):
+        assert np.array_equal(a, b)
+    xf = inp.all_inputs("float32", 4, n, m)
+    od = replay.replay(pd, xf, "float32", cnt, chunk_bytes=256, instances=2, K=1, sched="random", seed=1)
+    os_ = replay.replay(ps, xf, "float32", cnt, chunk_bytes=256, instances=2, K=1)
+    for a, b in zip(od, os_):
+        assert np.array_equal(a.view(np.uint8), b.view(np.uint8))
+    for n_mb, K in ((1, 1), (2, 1), (3, 2)):
+        for inplace in (False, True):
+            assert replay.happens_before_races(pd, n_mb=n_mb, instances=1, K=K, inplace=inplace) == []
+    assert replay.deadlock_free(pd, Ks=(1,), n_mbs=(1, 2, 3, 16))
+
+
+def test_direct_race_checker_catches_missing_ack_dependency():
+    """Mutation: dropping the pull-send acknowledgement dependencies lets a later write
+    of the sender's location race with the peer's pull -- the I2 checker must see it."""
+    # rank 1 pulls <0,0> (rrc, step 0); rank 2 then overwrites <0,0> (recv, step 1) with a
+    # value that does not depend on that read: only the ack dependency orders them
+    # (in-place: the pulled send-buffer copy and the pushed receive-buffer copy alias)
+    g = ir.IR("x", "allreduce", 3, 3, [ir.Transfer(0, 1, 0, 0, "rrc"), ir.Transfer(2, 0, 1, 0, "recv")])
+    pd = lower.lower(g, "pair", direct=True)
+    assert replay.happens_before_races(pd, n_mb=2, instances=1, K=1, inplace=True) == []
+    assert any(p.ack_deps for r in pd.prims for p in pd.prims[r])
+    for r in pd.prims:
+        for p in pd.prims[r]:
+            p.ack_deps = []
+    assert replay.happens_before_races(pd, n_mb=2, instances=1, K=1, inplace=True) != []

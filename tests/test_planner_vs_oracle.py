@@ -54,12 +54,13 @@ def _norm_oracle(pl):
             return (p.kind, p.chunk, p.pc,
                     tuple(tasks[p.recv_task]) if p.recv_task is not None else None,
                     tuple(tasks[p.send_task]) if p.send_task is not None else None,
-                    p.src_buf or "none", p.dst_buf or "none", p.has_counter)
+                    p.src_buf or "none", p.dst_buf or "none", p.has_counter, p.rem_buf or "none")
 
         ctas = []
         for sl, rl in pl.lanes[r]:
             ctas.append(tuple(
-                tuple((key(prims[i]), tuple(sorted(key(prims[d]) for d in prims[i].deps))) for i in lane)
+                tuple((key(prims[i]), tuple(sorted(key(prims[d]) for d in prims[i].deps)),
+                       tuple(sorted(key(prims[d]) for d in prims[i].ack_deps))) for i in lane)
                 for lane in (sl, rl)))
         out.append(dict(
             ctas=ctas, n_conn=pl.n_connections[r], paper_tbs=pl.paper_tbs(r),
@@ -79,12 +80,13 @@ def _norm_cpp(js):
             return (p["kind"], p["chunk"], p["pc"],
                     tasks[p["recv_task"]] if p["recv_task"] >= 0 else None,
                     tasks[p["send_task"]] if p["send_task"] >= 0 else None,
-                    p["src"], p["dst"], p["counter"])
+                    p["src"], p["dst"], p["counter"], p["rem"])
 
         ctas = []
         for c in rp["ctas"]:
             ctas.append(tuple(
-                tuple((key(prims[i]), tuple(sorted(key(prims[d]) for d in prims[i]["deps"]))) for i in lane)
+                tuple((key(prims[i]), tuple(sorted(key(prims[d]) for d in prims[i]["deps"])),
+                       tuple(sorted(key(prims[d]) for d in prims[i]["ack_deps"]))) for i in lane)
                 for lane in (c["send"], c["recv"])))
         out.append(dict(ctas=ctas, n_conn=rp["n_connections"], paper_tbs=rp["paper_tbs"],
                         send_groups=rp["send_groups"], recv_groups=rp["recv_groups"]))
@@ -210,3 +212,18 @@ def test_round_robin_plan_matches_oracle(name, coll, n, kw):
     tasks = [tuple(t) for t in js["plan"]["tasks"]]
     assert [[tasks[i] for i in pc] for pc in js["plan"]["Pr"]] == [[tuple(g.transfers[i]) for i in pc] for pc in pr]
     assert _norm_cpp(js) == _norm_oracle(lower.lower(g, "pair", Pr=pr))
+
+
+@pytest.mark.parametrize("name,coll,n,kw", CASES)
+@pytest.mark.parametrize("model", ["pair", "port"])
+def test_direct_plan_matches_oracle(name, coll, n, kw, model):
+    """Direct transport (R23): identical lowering (push/pull kinds, remote buffers, ack
+    dependencies) in the C++ planner and the oracle, and the same deadlock verdicts."""
+    g = _oracle_ir(name, coll, n, kw)
+    js = R.rescclPlanIr(g.to_text(), f"linkmodel={model} direct=1")
+    pl = lower.lower(g, model, direct=True)
+    assert js["plan"]["direct"] is True and pl.direct
+    assert _norm_cpp(js) == _norm_oracle(pl)
+    for K, nmb in ((1, 1), (1, 3), (2, 16)):
+        assert R.rescclCheckDeadlock(g.to_text(), f"linkmodel={model} direct=1", K, nmb) == \
+            replay.deadlock_free(pl, Ks=(K,), n_mbs=(nmb,))
