@@ -372,9 +372,17 @@ def main():
                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}, burst)",
                 "algorithmic_bytes_per_launch": int(algo_bytes),
                 "dram_algorithmic_bytes_per_launch": int(5.0 * (nr - 1) / nr * S * nr)}
-    tr = os.environ.get("RESCCL_BENCH_TRAFFIC")
-    if tr:
-        roof["traffic"] = float(tr)
+    # measured DRAM traffic of this exact workload from a committed ncu capture (if any)
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            tr = json.load(f)
+        key = (f"{args.algo}/{n}/{S}/{args.dtype}/{'direct' if info.get('direct') else 'staged'}/"
+               f"{info['instances']}/{info['chunkbytes']}")
+        if key in tr:
+            roof["traffic"] = tr[key]["traffic"]
+            roof["traffic_source"] = tr[key]["source"]
+    except Exception:
+        pass
 
     cpu = None
     if not args.no_cpu_baseline and not multi:

@@ -14,7 +14,7 @@ import torch
 import paper_conf_sigcomm_liuhlgcwz025_b200 as R
 
 N = 8
-BASE = dict(instances=18, chunkbytes=4 << 20, fifodepth=2)
+BASE = dict(instances=18, chunkbytes=8 << 20, fifodepth=2, direct=int(os.environ.get("SWEEP_DIRECT", "1")))
 ELT = {"bfloat16": 2, "float32": 4, "int32": 4}
 
 
@@ -61,7 +61,7 @@ def measure(name, coll, gopts, opts, S, dtype="bfloat16", iters=10, warm=3):
                 "us": round(ms * 1e3, 2), "algbw_gbs": round(alg, 2), "busbw_gbs": round(bus, 2),
                 "ctas_per_rank": info["ctas"], "blocks": sum(info["blocks_per_rank"]),
                 "instances": info["instances"], "linkmodel": info["linkmodel"], "fused": info["plan"]["fused"],
-                "sched": info.get("sched"), "err": err}
+                "sched": info.get("sched"), "direct": info.get("direct"), "err": err}
     finally:
         grp.destroy()
 
