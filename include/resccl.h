@@ -159,6 +159,15 @@ rescclResult_t rescclReduceScatter(const void* sendbuf, void* recvbuf, size_t re
  * Writes IR text; size protocol as above. */
 rescclResult_t rescclGenerateIr(const char* name, rescclColl_t coll, int nranks, const char* opts, char* text,
                                 size_t* len);
+/* ResCCLang front end (BNF Fig. 14): execute a `def ResCCLAlgo(...):`
+ * program -- e.g. the paper's Fig. 16 listing -- and write the resulting IR text.
+ * rescclLoadAlgorithm / rescclPlanIr also accept such programs directly.
+ * InvalidUsage on syntax errors (message names the line). */
+rescclResult_t rescclParseResCCLang(const char* program, char* irText, size_t* len);
+/* Workflow phase timings (Fig. 10a): Parsing, Analysis (DAG),
+ * Scheduling (HPDS / RR), Lowering (translation, TB allocation, rank-0 kernel source)
+ * and, if `verify`, the blocking-model deadlock check; JSON with counts and ms. */
+rescclResult_t rescclProfilePlanner(const char* program, const char* opts, int verify, char* json, size_t* len);
 /* Plan an IR (header keys as for rescclLoadAlgorithm; `opts` overrides them) and
  * write the plan JSON. */
 rescclResult_t rescclPlanIr(const char* irText, const char* opts, char* json, size_t* len);

@@ -45,7 +45,7 @@ EXPORTS = [
     "rescclLoadAlgorithm", "rescclSetActiveAlgorithm", "rescclGetPlanInfo", "rescclGetTbUtilization",
     "rescclAllReduce",
     "rescclAllGather", "rescclReduceScatter", "rescclGenerateIr", "rescclPlanIr",
-    "rescclCodegenIr", "rescclCompileIr", "rescclCheckDeadlock",
+    "rescclCodegenIr", "rescclCompileIr", "rescclCheckDeadlock", "rescclParseResCCLang", "rescclProfilePlanner",
 ]
 
 _c = ctypes
@@ -74,6 +74,8 @@ _SIGS = {
     "rescclCodegenIr": (_i, [_c.c_char_p, _c.c_char_p, _i, _i, _c.c_char_p, _c.POINTER(_sz)]),
     "rescclCompileIr": (_i, [_c.c_char_p, _c.c_char_p, _i, _i, _c.POINTER(_sz)]),
     "rescclCheckDeadlock": (_i, [_c.c_char_p, _c.c_char_p, _i, _i, _c.POINTER(_i)]),
+    "rescclParseResCCLang": (_i, [_c.c_char_p, _c.c_char_p, _c.POINTER(_sz)]),
+    "rescclProfilePlanner": (_i, [_c.c_char_p, _c.c_char_p, _i, _c.c_char_p, _c.POINTER(_sz)]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -100,9 +102,16 @@ def _b(s):
 def _sized(fn, *args) -> str:
     n = _sz(0)
     _check(fn(*args, None, _c.byref(n)), fn.__name__)
-    buf = _c.create_string_buffer(n.value)
-    _check(fn(*args, buf, _c.byref(n)), fn.__name__)
-    return buf.value.decode()
+    for _ in range(4):  # outputs with timings may grow between the two calls
+        cap = n.value + 4096
+        buf = _c.create_string_buffer(cap)
+        n = _sz(cap)
+        rc = fn(*args, buf, _c.byref(n))
+        if rc == rescclInvalidArgument and n.value > cap:
+            continue
+        _check(rc, fn.__name__)
+        return buf.value.decode()
+    _check(rc, fn.__name__)
 
 
 # ------------------------------------------------------------------ C-ABI wrappers (same names)
@@ -214,6 +223,14 @@ def rescclReduceScatter(sendbuf: int, recvbuf: int, recvcount: int, dtype: int, 
 
 def rescclGenerateIr(name: str, coll: str, nranks: int, opts: str = "") -> str:
     return _sized(_lib.rescclGenerateIr, _b(name), COLLS[coll], nranks, _b(opts))
+
+
+def rescclParseResCCLang(program: str) -> str:
+    return _sized(_lib.rescclParseResCCLang, _b(program))
+
+
+def rescclProfilePlanner(program: str, opts: str = "", verify: bool = False) -> dict:
+    return json.loads(_sized(_lib.rescclProfilePlanner, _b(program), _b(opts), int(verify)))
 
 
 def rescclPlanIr(ir_text: str, opts: str = "") -> dict:

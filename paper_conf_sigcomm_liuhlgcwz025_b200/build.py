@@ -29,6 +29,7 @@ SOURCES = [
     "plan/ir.cc",
     "plan/plan.cc",
     "plan/codegen.cc",
+    "plan/rescclang.cc",
     "comm/comm.cc",
 ]
 HEADERS = [

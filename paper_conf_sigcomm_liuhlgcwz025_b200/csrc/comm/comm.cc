@@ -12,6 +12,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -390,11 +391,24 @@ size_t arena_default() {
   return v ? (size_t)atoll(v) : (size_t)128 << 20;
 }
 
+// IR text, or a ResCCLang program (`def ResCCLAlgo(...):`, Fig. 14/16)
+Ir parse_any(const std::string& text) {
+  std::istringstream is(text);
+  std::string line;
+  while (std::getline(is, line)) {  // first non-blank, non-comment line decides
+    size_t i = line.find_first_not_of(" \t\r");
+    if (i == std::string::npos || line[i] == '#') continue;
+    if (line.compare(i, 4, "def ") == 0) return parse_rescclang(text);
+    break;
+  }
+  return parse_ir(text);
+}
+
 std::shared_ptr<AlgoShared> build_algo(const std::string& text, int nranks) {
   auto a = std::make_shared<AlgoShared>();
   a->text = text;
   try {
-    a->ir = parse_ir(text);
+    a->ir = parse_any(text);
   } catch (PlanError& e) {
     fail(rescclInvalidUsage, std::string("IR: ") + e.what());
   }
@@ -740,7 +754,7 @@ Group* make_group(int dev, int n) {
 
 Plan plan_from(const char* irText, const char* opts, Options* o_out, Ir* ir_out) {
   if (!irText) fail(rescclInvalidArgument, "irText is NULL");
-  Ir ir = parse_ir(irText);
+  Ir ir = parse_any(irText);
   Options o = make_options(ir, opts);
   Plan p = make_plan(ir, o);
   if (o_out) *o_out = o;
@@ -1096,6 +1110,51 @@ rescclResult_t rescclGenerateIr(const char* name, rescclColl_t coll, int nranks,
   for (auto& kv : parse_kv(opts)) o[kv.first] = to_long(kv.second, kv.first);
   Ir ir = generate(name, (Coll)coll, nranks, o);
   write_out(ir.to_text(), text, len);
+  API_END
+}
+
+rescclResult_t rescclProfilePlanner(const char* program, const char* opts, int verify, char* json, size_t* len) {
+  API_BEGIN
+  if (!program) fail(rescclInvalidArgument, "program is NULL");
+  using clk = std::chrono::steady_clock;
+  auto ms = [](clk::time_point a, clk::time_point b) {
+    return std::chrono::duration<double, std::milli>(b - a).count();
+  };
+  auto t0 = clk::now();
+  Ir ir = parse_any(program);                       // Parsing
+  auto t1 = clk::now();
+  Options o = make_options(ir, opts);
+  Dag d = build_dag(ir);                            // Analysis
+  auto t2 = clk::now();
+  auto pr = o.sched ? round_robin(ir, d, o.model) : hpds(ir, d, o.model);  // Scheduling
+  auto t3 = clk::now();
+  Plan p = lower(ir, o.model, false, &pr, o.direct != 0);  // Lowering (translation + TB allocation)
+  Layout L = make_layout(p, o.fifo_depth, o.instances, o.chunk_bytes);
+  CodegenOpts co;
+  co.rank_lo = 0;
+  co.rank_hi = 1;
+  co.nwarps = o.nwarps;
+  std::string src = codegen(p, L, co);              // kernel source of rank 0
+  auto t4 = clk::now();
+  bool ok = true;
+  if (verify) ok = deadlock_free(p, 1, 2);
+  auto t5 = clk::now();
+  int max_cta = 0;
+  for (auto& r : p.ranks) max_cta = std::max(max_cta, (int)r.ctas.size());
+  std::ostringstream out;
+  out << "{\"nranks\":" << ir.nranks << ",\"tasks\":" << ir.t.size() << ",\"edges\":" << d.edges.size()
+      << ",\"subpipelines\":" << pr.size() << ",\"max_ctas_per_rank\":" << max_cta
+      << ",\"parse_ms\":" << ms(t0, t1) << ",\"analysis_ms\":" << ms(t1, t2) << ",\"schedule_ms\":" << ms(t2, t3)
+      << ",\"lower_ms\":" << ms(t3, t4) << ",\"verify_ms\":" << ms(t4, t5)
+      << ",\"deadlock_free\":" << (ok ? "true" : "false") << ",\"rank0_src_bytes\":" << src.size() << "}";
+  write_out(out.str(), json, len);
+  API_END
+}
+
+rescclResult_t rescclParseResCCLang(const char* program, char* irText, size_t* len) {
+  API_BEGIN
+  if (!program) fail(rescclInvalidArgument, "program is NULL");
+  write_out(parse_rescclang(program).to_text(), irText, len);
   API_END
 }
 

@@ -70,4 +70,8 @@ Ir generate(const std::string& name, Coll coll, int n, const std::map<std::strin
 
 uint64_t splitmix64(uint64_t x);
 
+// ResCCLang front end (BNF Fig. 14): executes a `def ResCCLAlgo(...):`
+// program (e.g. the Fig. 16 listing) and returns its transfer IR.  Throws PlanError.
+Ir parse_rescclang(const std::string& program);
+
 }  // namespace resccl

@@ -100,10 +100,12 @@ Dag build_dag(const Ir& ir) {
   }
   Dag d;
   d.preds.assign(T, {});
+  d.succs.assign(T, {});
   for (auto& kv : er) {
     d.edges.push_back(kv.first);
     d.edge_ranks.emplace_back(kv.second.begin(), kv.second.end());
     d.preds[kv.first.second].push_back(kv.first.first);
+    d.succs[kv.first.first].push_back(kv.first.second);
   }
   return d;
 }
@@ -121,46 +123,37 @@ static void task_links(const Transfer& x, LinkModel m, int n, LinkKey out[2], in
   }
 }
 
-template <class PickChunk>
+// Incremental list scheduler: per-chunk ready sets ordered by (step, src, dst) and a
+// remaining-predecessor count per task, so a task becomes ready right after its last
+// predecessor leaves G (R4: before the next inner iteration).  Alg. 1's chunk choice
+// (line 9) uses an ordered set of (priority, ChunkId).  O(T log T + #Pc * C log C).
 static std::vector<std::vector<int>> list_schedule(const Ir& ir, const Dag& dag, LinkModel m, bool rr) {
   const int T = (int)ir.t.size(), N = ir.nranks;
-  std::vector<char> inG(T, 1);
-  int left = T;
-  std::vector<int> chunks;
-  {
-    std::set<int> cs;
-    for (auto& x : ir.t) cs.insert(x.chunk);
-    chunks.assign(cs.begin(), cs.end());
+  auto cmp = [&](int a, int b) {
+    auto& x = ir.t[a];
+    auto& y = ir.t[b];
+    return std::tie(x.step, x.src, x.dst, a) < std::tie(y.step, y.src, y.dst, b);
+  };
+  std::map<int, std::set<int, decltype(cmp)>> ready;
+  std::vector<int> npred(T);
+  std::set<int> chunkset;
+  for (auto& x : ir.t) chunkset.insert(x.chunk);
+  std::vector<int> chunks(chunkset.begin(), chunkset.end());
+  for (int c : chunks) ready.emplace(c, std::set<int, decltype(cmp)>(cmp));
+  for (int i = 0; i < T; ++i) {
+    npred[i] = (int)dag.preds[i].size();
+    if (npred[i] == 0) ready.at(ir.t[i].chunk).insert(i);
   }
-  std::map<int, std::vector<int>> tasks_of;
-  for (int i = 0; i < T; ++i) tasks_of[ir.t[i].chunk].push_back(i);
   std::map<int, int> prio;
   for (int c : chunks) prio[c] = 0;
+  int left = T;
   std::vector<std::vector<int>> Pr;
-
-  auto ready_of = [&](int C) {
-    std::vector<int> ready;
-    for (int i : tasks_of[C]) {
-      if (!inG[i]) continue;
-      bool ok = true;
-      for (int p : dag.preds[i])
-        if (inG[p]) { ok = false; break; }
-      if (ok) ready.push_back(i);
-    }
-    std::sort(ready.begin(), ready.end(), [&](int a, int b) {
-      auto& x = ir.t[a];
-      auto& y = ir.t[b];
-      return std::tie(x.step, x.src, x.dst) < std::tie(y.step, y.src, y.dst);
-    });
-    return ready;
-  };
-
   while (left > 0) {                                   // line 5
     std::vector<int> pc;                               // line 6
     std::set<LinkKey> used;
     auto take = [&](int C) {                           // lines 10-15: NodeList of chunk C
       std::vector<int> nl;
-      for (int i : ready_of(C)) {
+      for (int i : ready.at(C)) {
         LinkKey lk[2];
         int nk;
         task_links(ir.t[i], m, N, lk, &nk);
@@ -174,21 +167,29 @@ static std::vector<std::vector<int>> list_schedule(const Ir& ir, const Dag& dag,
       }
       return nl;
     };
+    auto remove = [&](const std::vector<int>& nl) {    // line 22: G.remove(NodeList)
+      for (int i : nl) {
+        ready.at(ir.t[i].chunk).erase(i);
+        --left;
+        for (int s : dag.succs[i])
+          if (--npred[s] == 0) ready.at(ir.t[s].chunk).insert(s);
+      }
+    };
     if (!rr) {
-      std::map<int, bool> F;                           // line 7
-      for (int c : chunks) F[c] = true;
-      while (true) {                                   // line 8
-        int C = -1;                                    // line 9: highest priority, lowest id
-        for (int c : chunks)
-          if (F[c] && (C < 0 || prio[c] > prio[C])) C = c;
-        if (C < 0) break;
+      // line 7: F = all true; line 9: highest priority, ties -> lowest ChunkId
+      std::set<std::pair<int, int>> Q;                 // (-priority, chunk) of flagged chunks
+      for (int c : chunks) Q.insert({-prio[c], c});
+      while (!Q.empty()) {                             // line 8
+        int C = Q.begin()->second;
         auto nl = take(C);
         if (nl.empty()) {
-          F[C] = false;                                // line 17
+          Q.erase(Q.begin());                          // line 17
         } else {
           pc.insert(pc.end(), nl.begin(), nl.end());   // line 19
+          Q.erase(Q.begin());
           prio[C] -= 1;                                // lines 20-21
-          for (int i : nl) { inG[i] = 0; --left; }     // line 22
+          Q.insert({-prio[C], C});
+          remove(nl);
         }
       }
     } else {                                           // RR baseline: fixed ascending order
@@ -199,7 +200,7 @@ static std::vector<std::vector<int>> list_schedule(const Ir& ir, const Dag& dag,
           auto nl = take(C);
           if (!nl.empty()) {
             pc.insert(pc.end(), nl.begin(), nl.end());
-            for (int i : nl) { inG[i] = 0; --left; }
+            remove(nl);
             progress = true;
           }
         }
@@ -211,12 +212,11 @@ static std::vector<std::vector<int>> list_schedule(const Ir& ir, const Dag& dag,
   return Pr;
 }
 
-struct NoPick {};
 std::vector<std::vector<int>> hpds(const Ir& ir, const Dag& dag, LinkModel m) {
-  return list_schedule<NoPick>(ir, dag, m, false);
+  return list_schedule(ir, dag, m, false);
 }
 std::vector<std::vector<int>> round_robin(const Ir& ir, const Dag& dag, LinkModel m) {
-  return list_schedule<NoPick>(ir, dag, m, true);
+  return list_schedule(ir, dag, m, true);
 }
 
 // ----------------------------------------------------------------------------- lowering

@@ -25,6 +25,7 @@ struct Dag {
   std::vector<std::pair<int, int>> edges;      // sorted (u, v)
   std::vector<std::vector<int>> edge_ranks;    // ranks of the inducing locations, per edge
   std::vector<std::vector<int>> preds;         // per task
+  std::vector<std::vector<int>> succs;         // per task
 };
 
 void validate_ir(const Ir& ir);            // I6; throws PlanError
