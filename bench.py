@@ -202,6 +202,8 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("RESCCL_BENCH_ONE_DEVICE") == "1":
+        local = 0  # test aid: every rank on cuda:0 (CUDA IPC between processes of one device)
     multi = world > 1
     if multi:
         import torch.distributed as dist
