@@ -85,7 +85,15 @@ __device__ __forceinline__ u64 globaltimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
-__device__ __forceinline__ void nanosleep_(u32 ns) { asm volatile("nanosleep.u32 %0;" ::"r"(ns)); }
+#ifndef RESCCL_BACKOFF
+#define RESCCL_BACKOFF 1
+#endif
+// polling back-off (RESCCL_BACKOFF=0: pure spin)
+__device__ __forceinline__ void nanosleep_(u32 ns) {
+#if RESCCL_BACKOFF
+  asm volatile("nanosleep.u32 %0;" ::"r"(ns));
+#endif
+}
 
 struct V4 {
   u32 x, y, z, w;

@@ -4,9 +4,10 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 import paper_conf_sigcomm_liuhlgcwz025_b200 as R
 N = 8
-for opts in ["instances=18 chunkbytes=4194304 fifodepth=2 tmamin=0", "instances=18 chunkbytes=4194304 fifodepth=2",
-             "instances=1 chunkbytes=4194304 fifodepth=2", "instances=4 chunkbytes=262144 fifodepth=2",
-             "instances=18 chunkbytes=4194304 fifodepth=2 tma=0"]:
+OPTS = sys.argv[1:] or ["instances=18 chunkbytes=8388608 direct=1", "instances=18 chunkbytes=8388608 direct=1 backoff=0",
+                        "instances=18 chunkbytes=8388608 direct=1 tma=0", "instances=18 chunkbytes=8388608 direct=1 tma=0 backoff=0",
+                        "instances=2 chunkbytes=8388608 direct=1 tma=0 backoff=0", "instances=18 chunkbytes=4194304 direct=0"]
+for opts in OPTS:
     text = R.rescclGenerateIr("ring", "allreduce", N)
     h, rest = text.split("\n", 1)
     grp = R.VirtualGroup(N, 0)

@@ -1,0 +1,69 @@
+"""Config C5 analogue on one B200: a bf16 GEMM loop on one stream, 25 MiB bf16 bucket
+AllReduces (ring, 8 virtual ranks, direct transport) on another; GEMM TFLOP/s alone vs
+concurrent, and AR time, for several SM budgets (instances -> 8 x instances CTAs)."""
+import json, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+
+N = 8
+M = int(sys.argv[1]) if len(sys.argv) > 1 else 8192
+a = torch.randn(M, M, device="cuda:0", dtype=torch.bfloat16)
+b = torch.randn(M, M, device="cuda:0", dtype=torch.bfloat16)
+c = torch.empty(M, M, device="cuda:0", dtype=torch.bfloat16)
+sg = torch.cuda.Stream()
+sc = torch.cuda.Stream()
+flops = 2 * M ** 3
+
+
+def gemm_loop(n):
+    with torch.cuda.stream(sg):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(sg)
+        for _ in range(n):
+            torch.matmul(a, b, out=c)
+        e1.record(sg)
+    return e0, e1
+
+
+for _ in range(3):
+    torch.matmul(a, b, out=c)
+torch.cuda.synchronize()
+e0, e1 = gemm_loop(40)
+torch.cuda.synchronize()
+alone = flops * 40 / (e0.elapsed_time(e1) * 1e-3) / 1e12
+print(json.dumps({"gemm_alone_tflops": round(alone, 1), "M": M}), flush=True)
+
+cnt = 25 * (1 << 20) // 2
+for inst in (1, 2, 4, 8, 18):
+    text = R.rescclGenerateIr("ring", "allreduce", N)
+    h, rest = text.split("\n", 1)
+    grp = R.VirtualGroup(N, 0)
+    grp.load(h + f" instances={inst} chunkbytes=4194304 direct=1\n" + rest)
+    s = [torch.randn(cnt, device="cuda:0").to(torch.bfloat16) for _ in range(N)]
+    r = [torch.empty_like(x) for x in s]
+    for _ in range(3):
+        grp.allreduce(s, r, stream=sc.cuda_stream)
+    torch.cuda.synchronize()
+    # AR alone
+    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    f0.record(sc)
+    for _ in range(40):
+        grp.allreduce(s, r, stream=sc.cuda_stream)
+    f1.record(sc)
+    torch.cuda.synchronize()
+    ar_alone = f0.elapsed_time(f1) / 40
+    # concurrent
+    g0, g1 = gemm_loop(40)
+    f0.record(sc)
+    for _ in range(40):
+        grp.allreduce(s, r, stream=sc.cuda_stream)
+    f1.record(sc)
+    torch.cuda.synchronize()
+    conc = flops * 40 / (g0.elapsed_time(g1) * 1e-3) / 1e12
+    ar_conc = f0.elapsed_time(f1) / 40
+    print(json.dumps({"instances": inst, "comm_ctas": N * inst, "gemm_concurrent_tflops": round(conc, 1),
+                      "gemm_slowdown_pct": round(100 * (1 - conc / alone), 2), "ar_alone_us": round(ar_alone * 1e3, 1),
+                      "ar_concurrent_us": round(ar_conc * 1e3, 1), "bucket_mib": 25,
+                      "err": grp.async_error()}), flush=True)
+    grp.destroy()
