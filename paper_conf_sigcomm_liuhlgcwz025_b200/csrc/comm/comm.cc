@@ -134,7 +134,7 @@ struct Options {
   int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
   int direct = 0;    // direct transport (R23): virtual ranks / single-process only
   int l2hint = 1;
-  int tma_min = 32768;
+  int tma_min = 163840;  // r01: register path wins below ~160 KiB slices (latency-bound)
   int backoff = 1;
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
 };
@@ -444,9 +444,13 @@ std::string info_json(const AlgoShared& a) {
   return o.str();
 }
 
-Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, int hi, bool gpu_scope) {
+// use_tma: the call's instance slices reach `tmamin` bytes; otherwise a variant without
+// the TMA engine (no dynamic shared memory, no mbarrier setup) is launched -- small
+// messages are latency-bound and the staging only costs launch overhead there.
+Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, int hi, bool gpu_scope,
+                 bool use_tma) {
   std::string key = std::to_string((int)dt) + "/" + std::to_string((int)op) + "/" + std::to_string(lo) + "-" +
-                    std::to_string(hi) + "/" + (gpu_scope ? "g" : "s");
+                    std::to_string(hi) + "/" + (gpu_scope ? "g" : "s") + (use_tma ? "/t" : "/n");
   auto it = a.kernels.find(key);
   if (it != a.kernels.end()) return it->second;
   CodegenOpts co;
@@ -454,7 +458,7 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.rank_hi = hi;
   co.gpu_scope = gpu_scope;
   co.nwarps = a.opt.nwarps;
-  co.tma = a.opt.tma;
+  co.tma = use_tma ? a.opt.tma : 0;
   co.tma_tile = a.opt.tma_tile;
   co.tma_stages = a.opt.tma_stages;
   co.trace = a.opt.trace;
@@ -600,7 +604,8 @@ void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const vo
   ka.err = comm->err_dev;
   ka.timeout_ns = timeout_ns();
   ka.trace = trace_buffer(a, a.lay.ctas[comm->rank] * a.opt.instances, ka.block_base);
-  Kern& k = get_kernel(a, c.dt, c.op, comm->rank, comm->rank + 1, false);
+  const bool use_tma = a.opt.tma && g.Mi * elt_size(c.dt) >= a.opt.tma_min;
+  Kern& k = get_kernel(a, c.dt, c.op, comm->rank, comm->rank + 1, false, use_tma);
   launch(k, a.lay.ctas[comm->rank] * a.opt.instances, 32 * a.opt.nwarps, ka, s);
   algo->mb_cum += (unsigned long long)g.n_mb;
 }
@@ -629,7 +634,8 @@ void group_launch(Group* G, Pending& p) {
   ka.err = G->err_dev;
   ka.timeout_ns = timeout_ns();
   ka.trace = trace_buffer(a, a.lay.total_pairs * a.opt.instances, 0);
-  Kern& k = get_kernel(a, c.dt, c.op, 0, G->nranks, true);
+  const bool use_tma = a.opt.tma && g.Mi * elt_size(c.dt) >= a.opt.tma_min;
+  Kern& k = get_kernel(a, c.dt, c.op, 0, G->nranks, true, use_tma);
   cudaStream_t ls = p.streams.back();
   // order the launch after every caller's stream, and every caller's stream after it
   std::vector<cudaStream_t> others;

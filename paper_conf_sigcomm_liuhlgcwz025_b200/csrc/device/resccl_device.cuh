@@ -903,7 +903,7 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
   if ((F & kDirect) && (((F & kSend) && (F & kPull)) || ((F & kRecv) && !(F & kPull))))
     return L.tid == 0 ? run_flags<F>(L, d, p) : true;
 #ifndef RESCCL_TMA_MIN
-#define RESCCL_TMA_MIN 32768
+#define RESCCL_TMA_MIN 163840
 #endif
 #if RESCCL_TMA
   // small slices are latency-bound: the register path saves two bulk-copy round trips

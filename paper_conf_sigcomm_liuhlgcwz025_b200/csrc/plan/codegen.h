@@ -46,7 +46,7 @@ struct CodegenOpts {
   int tma_stages = 4;            // tiles in flight per lane
   int trace = 0;                 // per-lane lifetime / wait timers (TB utilisation, Table 3)
   int l2hint = 1;                // L2 evict_last on FIFO writes, evict_first on streams
-  int tma_min = 32768;           // slices below this many bytes use the register path
+  int tma_min = 163840;          // slices below this many bytes use the register path
   int backoff = 1;               // nanosleep back-off while polling flags
   int prefetch = 0;              // micro-batches of local operand prefetched into L2 ahead (off: r01)
 };

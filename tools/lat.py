@@ -13,7 +13,7 @@ for opts in OPTS:
     grp = R.VirtualGroup(N, 0)
     grp.load(h + " " + opts + "\n" + rest)
     res = {}
-    for S in [1024, 65536, 1 << 20, 4 << 20, 16 << 20]:
+    for S in [int(x) for x in os.environ.get('LAT_SIZES', str([1024, 65536, 1 << 20, 4 << 20, 16 << 20]))[1:-1].split(',')]:
         cnt = S // 2
         s = [torch.randn(cnt, device="cuda:0").to(torch.bfloat16) for _ in range(N)]
         r = [torch.empty_like(x) for x in s]
@@ -21,9 +21,9 @@ for opts in OPTS:
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        for _ in range(20): grp.allreduce(s, r)
+        for _ in range(10): grp.allreduce(s, r)
         e1.record(); torch.cuda.synchronize()
-        res[S] = round(e0.elapsed_time(e1) / 20 * 1e3, 1)
+        res[S] = round(e0.elapsed_time(e1) / 10 * 1e3, 1)
     # empty kernel-ish baseline: count=1
     print(json.dumps({"opts": opts, "us": res}), flush=True)
     grp.destroy()
