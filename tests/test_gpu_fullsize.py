@@ -69,3 +69,56 @@ def test_fullsize_sampled(algo, n, size_mb, dtype, opts):
                 assert np.array_equal(got.view(np.uint8), exp[r][c].view(np.uint8)), (r, c)
     finally:
         grp.destroy()
+
+
+@pytest.mark.timeout(600)
+@pytest.mark.parametrize("name,coll,gkw,size_mb,dtype,opts", [
+    ("ring", "allgather", {}, 1024, "bfloat16", dict(instances=18, chunkbytes=8 << 20, direct=1)),
+    ("synth", "reducescatter", {"seed": 0, "fanout": 2}, 256, "float32", dict(instances=4, chunkbytes=1 << 20)),
+    ("hm", "allreduce", {"g": 4}, 256, "bfloat16", dict(instances=4, chunkbytes=4 << 20, direct=1)),
+])
+def test_fullsize_sampled_ag_rs(name, coll, gkw, size_mb, dtype, opts):
+    """Sampled parity at C2/C3/C4 sizes for AllGather (total output) and ReduceScatter
+    (total input) and the hierarchical AllReduce in direct mode."""
+    import torch
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    n = 8
+    elt = {"bfloat16": 2, "float16": 2, "float32": 4}[dtype]
+    total = size_mb * (1 << 20) // elt
+    cnt = total if coll == "allreduce" else total // n     # per-rank count argument
+    send_n = cnt * n if coll == "reducescatter" else cnt
+    recv_n = cnt * n if coll == "allgather" else cnt
+    g = oir.generate(name, coll, n, **gkw)
+    for k, v in opts.items():
+        g.extra[k] = str(v)
+    grp = R.VirtualGroup(n, 0)
+    try:
+        grp.load(g.to_text())
+        sends = [inp.rank_input_torch(dtype, 13, r, send_n) for r in range(n)]
+        recvs = [torch.full((recv_n,), float("nan"), device="cuda:0", dtype=sends[0].dtype) for _ in range(n)]
+        getattr(grp, coll)(sends, recvs)
+        torch.cuda.synchronize()
+        assert grp.async_error() == 0
+        geo = replay.Geometry(coll, n, cnt, elt, opts["chunkbytes"], opts["instances"])
+        rng = np.random.default_rng(1)
+        pos = [_positions(geo, c, rng) for c in range(n)]
+        chunk_in = []
+        for r in range(n):
+            row = []
+            for c in range(n):
+                if coll == "allgather":
+                    row.append(inp.rank_input_at(dtype, 13, r, pos[c]) if r == c else None)
+                else:
+                    row.append(inp.rank_input_at(dtype, 13, r, geo.chunk_off("send", c) + pos[c]))
+            chunk_in.append(row)
+        exp = replay.dataflow_values(g, chunk_in, dtype)
+        for r in range(n):
+            for c in range(n):
+                if coll == "reducescatter" and c != r:
+                    continue
+                idx = torch.from_numpy(geo.chunk_off("recv", c) + pos[c]).to(recvs[r].device)
+                got = recvs[r][idx].cpu()
+                got = got.view(torch.int16).numpy().view(np.uint16) if dtype == "bfloat16" else got.numpy()
+                assert np.array_equal(got.view(np.uint8), exp[r][c].view(np.uint8)), (r, c)
+    finally:
+        grp.destroy()
