@@ -136,6 +136,7 @@ struct Options {
   int l2hint = 1;
   int tma_min = 163840;  // r01: register path wins below ~160 KiB slices (latency-bound)
   int backoff = 1;
+  int jitter = 0;
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
 };
 
@@ -179,6 +180,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "tmamin") o.tma_min = (int)to_long(v, k);
   else if (k == "direct") o.direct = (int)to_long(v, k);
   else if (k == "backoff") o.backoff = (int)to_long(v, k);
+  else if (k == "jitter") o.jitter = (int)to_long(v, k);
   else if (k == "sched") {
     if (v == "hpds") o.sched = 0;
     else if (v == "rr") o.sched = 1;
@@ -199,7 +201,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -466,6 +468,7 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.prefetch = a.opt.prefetch;
   co.tma_min = a.opt.tma_min;
   co.backoff = a.opt.backoff;
+  co.jitter = a.opt.jitter;
   std::string src = codegen(a.plan, a.lay, co);
   if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
     if (FILE* f = fopen((std::string(dump) + "_" + a.ir.name + "_" + coll_name(a.ir.coll) + ".cu").c_str(), "w")) {
@@ -1199,6 +1202,7 @@ rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo
   co.prefetch = o.prefetch;
   co.tma_min = o.tma_min;
   co.backoff = o.backoff;
+  co.jitter = o.jitter;
   write_out(codegen(p, L, co), src, len);
   API_END
 }
@@ -1221,6 +1225,7 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
   co.prefetch = o.prefetch;
   co.tma_min = o.tma_min;
   co.backoff = o.backoff;
+  co.jitter = o.jitter;
   co.gpu_scope = true;
   auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, true);
   if (cubin_bytes) *cubin_bytes = cub.size();

@@ -71,7 +71,7 @@ enum : int { kErrTimeout = 7 };
 #define RESCCL_SC ".sys"
 #endif
 
-__device__ __forceinline__ u64 ld_acquire(const u64* p) {
+__device__ __forceinline__ u64 ld_acquire_raw(const u64* p) {
   u64 v;
   asm volatile("ld.acquire" RESCCL_SC ".global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
@@ -79,7 +79,33 @@ __device__ __forceinline__ u64 ld_acquire(const u64* p) {
 __device__ __forceinline__ void st_relaxed(u64* p, u64 v) {
   asm volatile("st.relaxed" RESCCL_SC ".global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
-__device__ __forceinline__ void fence_release() { asm volatile("fence.acq_rel" RESCCL_SC ";" ::: "memory"); }
+#ifndef RESCCL_JITTER
+#define RESCCL_JITTER 0
+#endif
+// Fault injector (RESCCL_JITTER=1, debug): a pseudo-random 0..~8 us delay before every
+// flag / credit / counter post and after every successful acquire, to shake out
+// memory-ordering bugs (SURVEY §5 race detection).
+__device__ __forceinline__ void jitter() {
+#if RESCCL_JITTER
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  unsigned x = (unsigned)(t ^ (t >> 17)) * 2654435761u + (unsigned)clock() + threadIdx.x * 40503u + blockIdx.x * 97u;
+  x ^= x >> 13;
+  const unsigned ns = (x % 4u == 0) ? (x >> 20) % 8192u : 0u;
+  if (ns) asm volatile("nanosleep.u32 %0;" ::"r"(ns));
+#endif
+}
+__device__ __forceinline__ void fence_release() {
+  jitter();
+  asm volatile("fence.acq_rel" RESCCL_SC ";" ::: "memory");
+}
+__device__ __forceinline__ u64 ld_acquire(const u64* p) {
+  const u64 v = ld_acquire_raw(p);
+#if RESCCL_JITTER
+  jitter();
+#endif
+  return v;
+}
 __device__ __forceinline__ u64 globaltimer() {
   u64 t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
