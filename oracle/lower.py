@@ -60,7 +60,8 @@ class Prim:
     ack_deps: List[int] = field(default_factory=list)  # direct: pull-sends completed by the peer's ack
     direct: bool = False
     pull: bool = False
-    rem_buf: Optional[str] = None     # direct: buffer of the peer location (push target / pull source)
+    rem_buf: Optional[str] = None     # direct: buffer of the peer location a pull reads
+    rem_out: Optional[str] = None     # direct: buffer of the peer location a push writes
     has_counter: bool = False
     pid: int = -1
 
@@ -71,7 +72,10 @@ class Prim:
         return (self.kind, self.chunk, self.pc, rt, st, self.src_buf, self.dst_buf)
 
 
-DIRECT_KIND = {("send", False): "dsend", ("send", True): "psend", ("recv", False): "drecv", ("rrc", True): "prrc"}
+DIRECT_FUSED = {("prrc", "psend"): "prrc_p", ("prrc", "dsend"): "prrc_d",
+                ("drecv", "psend"): "drecv_p", ("drecv", "dsend"): "drecv_d"}
+PULL_SENDS = ("psend", "prrc_p", "drecv_p")      # outgoing task pulled: post "readable" only
+PUSH_RECVS = ("drecv", "drecv_p", "drecv_d")     # incoming payload pushed into our location
 
 
 FUSED_KIND = {  # (recv op, store) -> fused name
@@ -143,9 +147,8 @@ def _greedy_merge(conns_act: Dict[Tuple[int, str], set]) -> List[List[Tuple[int,
 def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool = False) -> Plan:
     """``direct`` (reading R23): no FIFO staging; recv tasks are pushed into the
     receiver's location after it posts "writable", rrc tasks are pulled from the
-    sender's location, whose completion is the receiver's read acknowledgement."""
-    if direct:
-        fuse = False
+    sender's location, whose completion is the receiver's read acknowledgement.
+    Fusion in direct mode chains a receive with the next hop's push or "readable"."""
     edges, edge_rank = build_dag(ir)
     check_defined_reads(ir)
     if Pr is None:
@@ -191,7 +194,7 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
             else:
                 s.direct = rv.direct = True
                 s.kind, rv.kind = "dsend", "drecv"
-                s.rem_buf = rv.dst_buf
+                s.rem_out = rv.dst_buf
                 rv.store = False
         rv.pid = len(prims[t.dst]); prims[t.dst].append(rv); recv_of[i] = (t.dst, rv.pid)
 
@@ -274,6 +277,12 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
                         break
                 store = (final and is_output(coll, r, a.chunk)) or readers != {t2}
                 a.send_task = t2
+                if direct:       # value stays in our location; the send part keeps its mode
+                    a.kind = DIRECT_FUSED[(a.kind, b.kind)]
+                    a.rem_out = b.rem_out
+                    if a.kind.startswith("drecv"):
+                        a.src_buf = a.dst_buf
+                    continue
                 a.store = store
                 a.kind = FUSED_KIND[(tasks[t1].op, store)]
                 if not store:
@@ -292,21 +301,28 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
             for k, p in enumerate(final_list):
                 if p.pid >= 0 and p.kind != "copy":
                     newid[p.pid] = k
+            raw_kind = {q.pid: q.kind for q in ps}
+
+            def is_ack(d):   # dependency on a pull-send: completes with the peer's ack
+                return direct and raw_kind[d] == "psend"
+
             for k, p in enumerate(final_list):
                 old = p.pid
                 p.pid = k
                 if p.kind == "copy":
                     continue
-                ds = set()
-                for d in deps[r][old]:
-                    ds.add(newid[remap[d]])
+                ds, acks = set(), set()
+                srcs = list(deps[r][old])
                 if old in fused_into.values():
                     for bpid, apid in fused_into.items():
                         if apid == old:
-                            for d in deps[r][bpid]:
-                                ds.add(newid[remap[d]])
+                            srcs += list(deps[r][bpid])
+                for d in srcs:
+                    (acks if is_ack(d) else ds).add(newid[remap[d]])
                 ds.discard(k)
+                acks.discard(k)
                 p.deps = sorted(ds)
+                p.ack_deps = sorted(acks)
             ncta = max(len(send_groups[r]), len(recv_groups[r]), 1)
             lane_lists = []
             for c in range(ncta):
@@ -315,12 +331,7 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
                 r_l = sorted((p for p in final_list if p.lane == "R" and p.cta == c),
                              key=lambda p: p.pc)
                 lane_lists.append(([p.pid for p in s_l], [p.pid for p in r_l]))
-            # direct: dependencies on pull-sends complete with the receiver's ack and are
-            # never implied by lane order
-            if direct:
-                for p in final_list:
-                    p.ack_deps = [d for d in p.deps if final_list[d].kind == "psend"]
-                    p.deps = [d for d in p.deps if final_list[d].kind != "psend"]
+            # (ack dependencies are never implied by lane order)
             # drop dependencies implied by lane order
             pos_in_lane = {}
             for c, (sl, rl) in enumerate(lane_lists):
@@ -347,11 +358,25 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
     plan._act = act
     if fuse and any(absorbed[r] for r in range(N)):
         from .replay import deadlock_free
+
+        def rebuilt(ab, fused):
+            op, ln = build(ab)
+            pl = Plan(ir, model, edges, edge_rank, Pr, pidx, op, ln, send_groups, recv_groups,
+                      {r: len(act[r]) for r in range(N)}, fused, direct)
+            pl._act = act
+            return pl
+
         if not deadlock_free(plan, Ks=(1,), n_mbs=(1, 2, 3, 16)):
-            out_prims, lanes = build({r: {} for r in range(N)})
-            plan = Plan(ir, model, edges, edge_rank, Pr, pidx, out_prims, lanes,
-                        send_groups, recv_groups, {r: len(act[r]) for r in range(N)}, False)
-            plan._act = act
+            # direct: fusions whose send part only posts "readable" add no wait edge
+            safe = {r: {b: a for b, a in absorbed[r].items() if prims[r][b].kind == "psend"}
+                    for r in range(N)} if direct else {r: {} for r in range(N)}
+            plan = None
+            if any(safe[r] for r in range(N)):
+                plan = rebuilt(safe, True)
+                if not deadlock_free(plan, Ks=(1,), n_mbs=(1, 2, 3, 16)):
+                    plan = None
+            if plan is None:
+                plan = rebuilt({r: {} for r in range(N)}, False)
     return plan
 
 

@@ -38,7 +38,7 @@ from typing import Dict, List, Optional, Tuple
 
 import numpy as np
 
-from .lower import Plan, conn_positions, is_output
+from .lower import PULL_SENDS, PUSH_RECVS, Plan, conn_positions, is_output
 from .numerics import combine
 
 ELT = {"int32": 4, "float32": 4, "float16": 2, "bfloat16": 2}
@@ -176,6 +176,17 @@ class _Sim:
                 return False
         return True
 
+    def send_ok(self, p, j, inst) -> bool:
+        if p.send_task is None:
+            return True
+        pos = self.pos(p.send_task, j)
+        cr = self.credit[(self._link(p.send_task), inst)]
+        if not p.direct:
+            return pos < cr + self.K
+        if p.kind in PULL_SENDS:                      # pull-send: post "readable"
+            return True
+        return cr >= pos + 1                          # push: receiver location writable
+
     def enabled(self, pr) -> bool:
         r, c, lane, inst, prog, k, j, phase = pr
         if k >= len(prog):
@@ -183,23 +194,17 @@ class _Sim:
         p = self.plan.prims[r][prog[k]]
         if p.kind == "copy":
             return True
-        if p.kind == "drecv" and phase == 1:          # push receiver waiting for the payload
-            return self.pos(p.recv_task, j) in self.fifo[(self._link(p.recv_task), inst)]
+        if p.kind in PUSH_RECVS and phase == 1:       # push receiver waiting for the payload
+            return (self.pos(p.recv_task, j) in self.fifo[(self._link(p.recv_task), inst)]
+                    and self.send_ok(p, j, inst))
         if not self.deps_ok(r, p, j, inst):
             return False
-        if p.recv_task is not None and p.kind != "drecv":
+        if p.kind in PUSH_RECVS:                      # phase 0: post "writable"
+            return True
+        if p.recv_task is not None:
             if self.pos(p.recv_task, j) not in self.fifo[(self._link(p.recv_task), inst)]:
                 return False
-        if p.send_task is not None:
-            pos = self.pos(p.send_task, j)
-            cr = self.credit[(self._link(p.send_task), inst)]
-            if not p.direct:
-                if pos >= cr + self.K:
-                    return False
-            elif not p.pull:                          # push: receiver location writable
-                if cr < pos + 1:
-                    return False
-        return True
+        return self.send_ok(p, j, inst)
 
     def finished(self) -> bool:
         return all(pr[5] >= len(pr[4]) for pr in self.procs)
@@ -207,7 +212,7 @@ class _Sim:
     def fire(self, pr, action=None):
         r, c, lane, inst, prog, k, j, phase = pr
         p = self.plan.prims[r][prog[k]]
-        if p.kind == "drecv" and phase == 0:          # post "writable", keep the micro-batch
+        if p.kind in PUSH_RECVS and phase == 0:       # post "writable", keep the micro-batch
             key = (self._link(p.recv_task), inst)
             self.credit[key] = max(self.credit[key], self.pos(p.recv_task, j) + 1)
             pr[7] = 1
@@ -222,7 +227,7 @@ class _Sim:
             if not p.direct:
                 assert pos == self.credit[key], "out-of-order consumption"
                 self.credit[key] += 1
-            elif p.pull:
+            elif p.kind not in PUSH_RECVS:            # pull: read acknowledged
                 self.credit[key] = max(self.credit[key], pos + 1)
         out = action(p, r, j, inst, incoming) if action else None
         if p.send_task is not None:
@@ -342,14 +347,14 @@ def replay(plan: Plan, inputs: List[np.ndarray], dtype: str, count: int, op: str
             return None
         lo, hi = g.slice(p.chunk, j, inst)
         tasks = plan.ir.transfers
-        if p.kind == "dsend":                         # direct push: write the receiver's location
+        if p.kind in ("dsend", "drecv_d"):            # direct push: write the receiver's location
             o = g.chunk_off(p.src_buf, p.chunk)
-            d, od = tasks[p.send_task].dst, g.chunk_off(p.rem_buf, p.chunk)
-            bufs[d][p.rem_buf][od + lo:od + hi] = bufs[r][p.src_buf][o + lo:o + hi]
+            d, od = tasks[p.send_task].dst, g.chunk_off(p.rem_out, p.chunk)
+            bufs[d][p.rem_out][od + lo:od + hi] = bufs[r][p.src_buf][o + lo:o + hi]
             return None
-        if p.kind in ("psend", "drecv"):              # flags only
+        if p.kind in ("psend", "drecv", "drecv_p"):   # flags only
             return None
-        if p.kind == "prrc":                          # direct pull: read the sender's location
+        if p.kind in ("prrc", "prrc_p", "prrc_d"):    # direct pull: read the sender's location
             s_, os_ = tasks[p.recv_task].src, g.chunk_off(p.rem_buf, p.chunk)
             incoming = bufs[s_][p.rem_buf][os_ + lo:os_ + hi].copy()
         if p.recv_task is None:                       # plain send
@@ -363,6 +368,12 @@ def replay(plan: Plan, inputs: List[np.ndarray], dtype: str, count: int, op: str
         if p.store:
             o = g.chunk_off(p.dst_buf, p.chunk)
             bufs[r][p.dst_buf][o + lo:o + hi] = v
+        if p.kind == "prrc_d":                        # ... and push it to the next hop
+            d, od = tasks[p.send_task].dst, g.chunk_off(p.rem_out, p.chunk)
+            bufs[d][p.rem_out][od + lo:od + hi] = v
+            return None
+        if p.kind == "prrc_p":
+            return None
         return v.copy() if p.send_task is not None else None
 
     sim.run(sched, seed, action)
@@ -404,34 +415,44 @@ def happens_before_races(plan: Plan, n_mb: int = 2, instances: int = 1, K: int =
         slink = sim._link(p.send_task) if p.send_task is not None else None
         rpos = sim.pos(p.recv_task, j) if p.recv_task is not None else None
         spos = sim.pos(p.send_task, j) if p.send_task is not None else None
-        if p.kind == "drecv" and phase == 1:
+        push_recv = p.kind in PUSH_RECVS
+
+        def send_joins():
+            if p.send_task is not None:
+                if not p.direct:
+                    if spos - K >= 0:
+                        join(credit_vc[(slink, inst, spos - K)])
+                elif p.kind not in PULL_SENDS:
+                    join(credit_vc[(slink, inst, spos)])
+
+        if push_recv and phase == 1:
             join(put_vc[(rlink, inst, rpos)])
+            send_joins()
         elif p.kind != "copy":
             for d in p.deps:
                 join(done_vc[(r, d, inst, j)])
             for d in p.ack_deps:
                 t = plan.prims[r][d].send_task
                 join(credit_vc[(sim._link(t), inst, sim.pos(t, j))])
-            if p.recv_task is not None and p.kind != "drecv":
-                join(put_vc[(rlink, inst, rpos)])
-            if p.send_task is not None:
-                if not p.direct:
-                    if spos - K >= 0:
-                        join(credit_vc[(slink, inst, spos - K)])
-                elif not p.pull:
-                    join(credit_vc[(slink, inst, spos)])
+            if not push_recv:
+                if p.recv_task is not None:
+                    join(put_vc[(rlink, inst, rpos)])
+                send_joins()
         jj = 0 if p.kind == "copy" else j
         if p.kind == "copy":
             acc.append(((r, "send", p.chunk, -1, -1), False))
             acc.append(((r, "recv", p.chunk, -1, -1), True))
-        elif p.kind == "dsend":
-            acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
-            acc.append(((tasks[p.send_task].dst, p.rem_buf, p.chunk, jj, inst), True))
-        elif p.kind == "prrc":
+        elif p.kind in ("dsend", "drecv_d"):
+            if not (push_recv and phase == 0):
+                acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
+                acc.append(((tasks[p.send_task].dst, p.rem_out, p.chunk, jj, inst), True))
+        elif p.kind in ("prrc", "prrc_p", "prrc_d"):
             acc.append(((tasks[p.recv_task].src, p.rem_buf, p.chunk, jj, inst), False))
             acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
             acc.append(((r, p.dst_buf, p.chunk, jj, inst), True))
-        elif p.kind not in ("psend", "drecv"):
+            if p.kind == "prrc_d":
+                acc.append(((tasks[p.send_task].dst, p.rem_out, p.chunk, jj, inst), True))
+        elif p.kind not in ("psend", "drecv", "drecv_p"):
             if p.recv_task is not None:
                 acc.append((("fifo", rlink, inst, rpos % K), False))
             if p.send_task is not None:
@@ -454,10 +475,10 @@ def happens_before_races(plan: Plan, n_mb: int = 2, instances: int = 1, K: int =
                 for jx in range(n_mb):
                     for ix in range(instances):
                         cells[(cell[0], cell[1], cell[2], jx, ix)].append((me, v[me], snap, w))
-        if p.kind == "drecv" and phase == 0:
+        if push_recv and phase == 0:
             credit_vc[(rlink, inst, rpos)] = snap          # "writable"
             return
-        if p.recv_task is not None and p.kind != "drecv":
+        if p.recv_task is not None and not push_recv:
             credit_vc[(rlink, inst, rpos)] = snap          # consumed / read acknowledged
         if p.send_task is not None:
             put_vc[(slink, inst, spos)] = snap             # payload / "written" / "readable"

@@ -58,8 +58,8 @@ struct KArgs {
   u64* trace;                         // RESCCL_TRACE: 4 x u64 per (block, lane), host-mapped
 };
 
-enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16, kDirect = 32, kPull = 64 };
-enum : int { BufSend = 0, BufRecv = 1, BufScratch = 2 };
+enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16, kDirect = 32, kPull = 64, kSendPull = 128 };
+enum : int { BufNone = -1, BufSend = 0, BufRecv = 1, BufScratch = 2 };
 enum : int { CollAllGather = 0, CollReduceScatter = 1, CollAllReduce = 2 };
 enum : int { OpSum = 0, OpMax = 1, OpMin = 2 };
 enum : int { kErrTimeout = 7 };
@@ -488,7 +488,8 @@ struct PrimDesc {
   i64 in_data, in_flag, in_cred, in_pos, in_n;
   i64 out_data, out_flag, out_cred, out_pos, out_n;
   i64 ctr;
-  int rem_rank, rem_buf;       // direct mode: the peer location (push target / pull source)
+  int rem_rank, rem_buf;       // direct mode: the peer location a pull reads
+  int out_rank, out_buf;       // direct mode: the peer location a push writes
   // dependency k is satisfied for micro-batch j when the u64 at deps[k] in this rank's
   // region reaches dep_n[k] * mb_base + dep_pos[k] * n_mb + j + 1: a completion counter
   // (n = 1, pos = 0) or, for a direct pull-send, the receiver's read credit of its link.
@@ -509,8 +510,17 @@ struct PrimPtrs {
   u64* out_flag;
   u64* out_cred;     // credit counter the receiver writes back (own arena)
   u64* ctr;
-  const char* R;     // direct mode: peer location base (chunk start)
+  const char* R;     // direct mode: pulled peer location base (chunk start)
+  char* Q;           // direct mode: pushed peer location base (chunk start)
   i64 len;           // chunk length (elements)
+};
+
+// primitive anatomy (compile-time, from the flags)
+template <int F> struct Kind {
+  static constexpr bool push_recv = (F & kDirect) && (F & kRecv) && !(F & kPull);  // payload pushed to us
+  static constexpr bool has_b = (F & kRecv) && !push_recv;             // incoming operand: FIFO slot / pulled
+  static constexpr bool send_data = (F & kSend) && !((F & kDirect) && (F & kSendPull));  // we write the payload
+  static constexpr int mf = (F & kReduce) | (has_b ? kRecv : 0);      // value = A (+) B, B, or A
 };
 
 __device__ __forceinline__ u64 dep_target(const KArgs& a, const PrimDesc& d, int k, int j) {
@@ -531,9 +541,16 @@ __device__ __forceinline__ void post_mb(const KArgs& a, const PrimDesc& d, const
   const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
   const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
   fence_release();
-  if (F & kSend) st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);
-  if (F & kRecv) st_relaxed(p.in_cred, in_seq + 1);
+  if (F & kSend) st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);   // payload / written / readable
+  if (Kind<F>::has_b) st_relaxed(p.in_cred, in_seq + 1);                        // consumed / read (push: posted earlier)
   if (d.ctr >= 0) st_relaxed(p.ctr, mb_base + j + 1);
+}
+
+template <int F>
+__device__ __forceinline__ void post_writable(const KArgs& a, const PrimDesc& d, const PrimPtrs& p, int j) {
+  const u64 in_seq = (u64)d.in_n * a.mb_base + (u64)d.in_pos * a.n_mb + j;
+  fence_release();
+  st_relaxed(p.in_cred, in_seq + 1);
 }
 
 // Non-blocking readiness of micro-batch j: local dependencies, payload, credit.
@@ -541,16 +558,17 @@ template <int F>
 __device__ __forceinline__ bool mb_ready(const Lane& L, const PrimDesc& d, const PrimPtrs& p, int j) {
   const KArgs& a = *L.a;
   const u64 mb_base = a.mb_base;
-  for (int k = 0; k < d.ndeps; ++k)
-    if (ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) < dep_target(a, d, k, j)) return false;
+  if (!Kind<F>::push_recv)  // (a push receiver checked its dependencies when it posted "writable")
+    for (int k = 0; k < d.ndeps; ++k)
+      if (ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) < dep_target(a, d, k, j)) return false;
   if (F & kRecv) {
     const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
     if (ld_acquire(p.in_flag + (in_seq % RESCCL_K)) < in_seq + 1) return false;
   }
   if (F & kSend) {
     const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
-    if (F & kDirect) {  // push: the receiver's location must be writable
-      if (ld_acquire(p.out_cred) < out_seq + 1) return false;
+    if (F & kDirect) {
+      if (!(F & kSendPull) && ld_acquire(p.out_cred) < out_seq + 1) return false;  // push: writable
     } else if (out_seq + 1 > (u64)RESCCL_K && ld_acquire(p.out_cred) < out_seq + 1 - RESCCL_K) {
       return false;
     }
@@ -571,12 +589,14 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
       bool ok = true;
       for (int k = 0; k < d.ndeps && ok; ++k)
         ok = L.wait_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, j));
+      if (ok && Kind<F>::push_recv) post_writable<F>(a, d, p, j);
       if (ok && (F & kRecv)) ok = L.wait_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1);
       if (ok && (F & kSend)) {
-        if (F & kDirect)
-          ok = L.wait_ge(p.out_cred, out_seq + 1);
-        else if (out_seq + 1 > (u64)RESCCL_K)
+        if (F & kDirect) {
+          if (!(F & kSendPull)) ok = L.wait_ge(p.out_cred, out_seq + 1);
+        } else if (out_seq + 1 > (u64)RESCCL_K) {
           ok = L.wait_ge(p.out_cred, out_seq + 1 - RESCCL_K);
+        }
       }
       if (!ok) *L.abort_flag = 1;
     }
@@ -586,11 +606,12 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
     slice_of(a, p.len, j, L.inst, lo, hi);
     const char* Aj = p.A ? p.A + lo * T::kSize : nullptr;
     char* D1j = p.D1 ? p.D1 + lo * T::kSize : nullptr;
-    const char* Bj = (F & kRecv) ? ((F & kDirect) ? p.R + lo * T::kSize : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT)
-                                 : nullptr;
-    char* D2j = (F & kSend) ? ((F & kDirect) ? (char*)p.R + lo * T::kSize : p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT)
-                            : nullptr;
-    move<T, OP, F & ~(kDirect | kPull), 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
+    const char* Bj = Kind<F>::has_b ? ((F & kDirect) ? p.R + lo * T::kSize
+                                                     : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT)
+                                    : nullptr;
+    char* D2j = Kind<F>::send_data ? ((F & kDirect) ? p.Q + lo * T::kSize : p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT)
+                                   : nullptr;
+    move<T, OP, Kind<F>::mf, 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
     L.sync();
     if (L.tid == 0) post_mb<F>(a, d, p, j);
   }
@@ -646,8 +667,20 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   const u64 pol_first = policy_evict_first();
   const u64 pol_last = policy_evict_last();
   int pf = 0;                 // next micro-batch whose local slice gets an L2 prefetch
+  int wp = 0;                 // push receiver (drecv_d): micro-batches posted "writable"
   while (pj < nmb) {
     bool prog = false;
+    if (Kind<F>::push_recv) {  // post "writable" as far ahead as the dependencies allow
+      while (wp < nmb) {
+        bool ok = true;
+        for (int k = 0; k < d.ndeps && ok; ++k)
+          ok = ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) >= dep_target(a, d, k, wp);
+        if (!ok) break;
+        post_writable<F>(a, d, p, wp);
+        ++wp;
+        prog = true;
+      }
+    }
 #if RESCCL_PREFETCH
     // (0) keep the local operand of the next RESCCL_PREFETCH micro-batches streaming into L2
     if (p.A && (F & (kReduce | kRecv)) != kRecv) {
@@ -660,7 +693,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
     }
 #endif
     // (1) readiness of the micro-batch the load cursor needs
-    if (rj < nmb && rj == lj && mb_ready<F>(L, d, p, rj)) {
+    if (rj < nmb && rj == lj && (!Kind<F>::push_recv || rj < wp) && mb_ready<F>(L, d, p, rj)) {
       fence_proxy_async();  // generic-proxy data (acquired) -> async-proxy reads
       ++rj;
       prog = true;
@@ -689,10 +722,10 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
         tma_load(sa + (u32)RESCCL_TMA_TILE, bsrc, nb, L.full + 8 * s, pol_first);
       } else {
         const char* src;
-        if (F & kRecv) {
+        if (Kind<F>::has_b) {  // staged receive: the FIFO slot
           const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + lj;
           src = p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off;
-        } else {
+        } else {               // send / pushed payload forwarded: our location
           src = p.A + lo_l * T::kSize + off;
         }
         mbar_expect_tx(L.full + 8 * s, nb);
@@ -719,9 +752,9 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       const u32 nb = (u32)((nb_s - off) < TB ? (nb_s - off) : TB);
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
       if (F & kStore) tma_store(p.D1 + lo_s * T::kSize + off, sa, nb, pol_first);
-      if (F & kSend) {
+      if (Kind<F>::send_data) {
         if (F & kDirect) {
-          tma_store((char*)p.R + lo_s * T::kSize + off, sa, nb, pol_first);
+          tma_store(p.Q + lo_s * T::kSize + off, sa, nb, pol_first);
         } else {
           const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + sj;
           tma_store(p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + off, sa, nb, pol_last);
@@ -743,14 +776,14 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       if (e0 < hi_h) {
         const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + pj;
         const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + pj;
-        const char* Bj = (F & kRecv) ? ((F & kDirect) ? p.R + e0 * T::kSize
-                                                     : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
-                                     : nullptr;
-        char* D2j = (F & kSend) ? ((F & kDirect) ? (char*)p.R + e0 * T::kSize
-                                                 : p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
-                                : nullptr;
+        const char* Bj = Kind<F>::has_b ? ((F & kDirect) ? p.R + e0 * T::kSize
+                                                         : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
+                                        : nullptr;
+        char* D2j = Kind<F>::send_data ? ((F & kDirect) ? p.Q + e0 * T::kSize
+                                                        : p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
+                                       : nullptr;
         for (i64 e = 0; e < hi_h - e0; ++e)
-          elem_move<T, OP>(F & ~(kDirect | kPull), p.A ? p.A + e0 * T::kSize : nullptr, Bj,
+          elem_move<T, OP>(Kind<F>::mf, p.A ? p.A + e0 * T::kSize : nullptr, Bj,
                            p.D1 ? p.D1 + e0 * T::kSize : nullptr, D2j, e);
       }
       fence_proxy_async();
@@ -830,16 +863,18 @@ __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const Prim
 // Direct-mode primitives that move no data (leader only): a pull-send posts "readable"
 // for each micro-batch once its dependencies hold; a push-receive posts "writable"
 // (credit) as soon as its dependencies hold -- running ahead of the payloads -- and
-// completes a micro-batch when the sender's "written" flag arrives.
+// completes a micro-batch when the sender's "written" flag arrives (drecv_p then also
+// posts "readable" for the next hop, which pulls from our location).
 template <int F>
 __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
   const KArgs& a = *L.a;
   const int nmb = a.n_mb;
   const u64 mb_base = a.mb_base;
-  int wp = 0, dj = 0;  // push-receive: writable posted / completed micro-batches
+  constexpr bool recv = F & kRecv;
+  int wp = 0, dj = 0;  // posted (readable / writable) / completed micro-batches
   u64 t_idle = 0;
   u32 spins = 0;
-  while ((F & kSend) ? wp < nmb : dj < nmb) {
+  while (recv ? dj < nmb : wp < nmb) {
     bool prog = false;
     if (wp < nmb) {
       bool ok = true;
@@ -847,7 +882,7 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
         ok = ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) >= dep_target(a, d, k, wp);
       if (ok) {
         fence_release();
-        if (F & kSend) {
+        if (!recv) {
           const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + wp;
           st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);
         } else {
@@ -858,10 +893,14 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
         prog = true;
       }
     }
-    if (!(F & kSend) && dj < wp) {
+    if (recv && dj < wp) {
       const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + dj;
       if (ld_acquire(p.in_flag + (in_seq % RESCCL_K)) >= in_seq + 1) {
         fence_release();
+        if (F & kSend) {  // drecv_p: the payload is in our location -> readable for the next hop
+          const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + dj;
+          st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);
+        }
         if (d.ctr >= 0) st_relaxed(p.ctr, mb_base + dj + 1);
         ++dj;
         prog = true;
@@ -903,7 +942,7 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
   p.len = chunk_len<RESCCL_COLL>(a, c);
   p.A = nullptr;
   p.D1 = nullptr;
-  if ((F & kCopy) || (F & kReduce) || !(F & kRecv))
+  if (d.src_buf != BufNone && ((F & kCopy) || (F & kReduce) || !Kind<F>::has_b))
     p.A = buf_ptr(a, L.rank, d.src_buf) + chunk_off<RESCCL_COLL>(d.src_buf, c, a.C) * T::kSize;
   if ((F & kCopy) || (F & kStore))
     p.D1 = buf_ptr(a, L.rank, d.dst_buf) + chunk_off<RESCCL_COLL>(d.dst_buf, c, a.C) * T::kSize;
@@ -924,16 +963,21 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
   p.out_flag = (F & kSend) ? at(peer, d.out_flag + (i64)L.inst * RESCCL_FLAGSTRIDE) : nullptr;
   p.out_cred = at(L.self, d.out_cred + (i64)L.inst * 128);
   p.ctr = at(L.self, d.ctr + (i64)L.inst * 128);
-  p.R = (F & kDirect) ? buf_ptr(a, d.rem_rank, d.rem_buf) + chunk_off<RESCCL_COLL>(d.rem_buf, c, a.C) * T::kSize
-                      : nullptr;
-  if ((F & kDirect) && (((F & kSend) && (F & kPull)) || ((F & kRecv) && !(F & kPull))))
-    return L.tid == 0 ? run_flags<F>(L, d, p) : true;
+  p.R = ((F & kDirect) && (F & kPull))
+            ? buf_ptr(a, d.rem_rank, d.rem_buf) + chunk_off<RESCCL_COLL>(d.rem_buf, c, a.C) * T::kSize
+            : nullptr;
+  p.Q = ((F & kDirect) && Kind<F>::send_data)
+            ? buf_ptr(a, d.out_rank, d.out_buf) + chunk_off<RESCCL_COLL>(d.out_buf, c, a.C) * T::kSize
+            : nullptr;
+  // no data moved here: pull-send, push-receive (+ readable for the next hop)
+  if ((F & kDirect) && !Kind<F>::has_b && !Kind<F>::send_data) return L.tid == 0 ? run_flags<F>(L, d, p) : true;
 #ifndef RESCCL_TMA_MIN
 #define RESCCL_TMA_MIN 163840
 #endif
 #if RESCCL_TMA
   // small slices are latency-bound: the register path saves two bulk-copy round trips
-  const unsigned long long al = (unsigned long long)p.A | (unsigned long long)p.D1 | (unsigned long long)p.R;
+  const unsigned long long al =
+      (unsigned long long)p.A | (unsigned long long)p.D1 | (unsigned long long)p.R | (unsigned long long)p.Q;
   if ((al & 15) == 0 && a.Mi * T::kSize >= RESCCL_TMA_MIN) {
     if (L.tid == 0) return pipe_leader<T, OP, F>(L, d, p);
     if (L.tid < 32) return true;

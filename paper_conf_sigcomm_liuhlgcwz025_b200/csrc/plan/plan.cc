@@ -13,8 +13,10 @@ namespace resccl {
 const char* Prim::kind_name() const {
   if (flags & kCopy) return "copy";
   if (flags & kDirect) {
-    if (flags & kSend) return (flags & kPull) ? "psend" : "dsend";
-    return (flags & kPull) ? "prrc" : "drecv";
+    if (!(flags & kRecv)) return (flags & kSendPull) ? "psend" : "dsend";
+    if (!(flags & kSend)) return (flags & kPull) ? "prrc" : "drecv";
+    if (flags & kPull) return (flags & kSendPull) ? "prrc_p" : "prrc_d";
+    return (flags & kSendPull) ? "drecv_p" : "drecv_d";
   }
   bool rv = flags & kRecv, sd = flags & kSend, red = flags & kReduce, st = flags & kStore;
   if (!rv) return "send";
@@ -294,7 +296,13 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
       bool store = (final_ && is_output(ir.coll, r, a.chunk)) || readers != std::set<int>{t2};
       a.send_task = t2;
       a.flags |= kSend;
-      if (!store) {
+      if (P.direct) {
+        // direct: the next hop pulls from / is pushed from our location, so the value
+        // stays stored; the send part keeps its push / pull mode
+        a.flags |= (b.flags & kSendPull);
+        a.rem_out = b.rem_out;
+        if (!(a.flags & kPull)) a.src_buf = a.dst_buf;  // push receiver forwards its location
+      } else if (!store) {
         a.flags &= ~kStore;
         a.dst_buf = BufNone;
       }
@@ -326,16 +334,24 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
       auto it = fused_into.find(raw_id);
       return newid.at(it == fused_into.end() ? raw_id : it->second);
     };
+    // direct mode: a dependency on a pull-send (also when absorbed into a fused prim)
+    // completes with the receiver's ack of that send's link -> ack dependency
+    auto is_ack = [&](int raw_id) {
+      return P.direct && (ps[raw_id].flags & kSendPull) && !(ps[raw_id].flags & kRecv);
+    };
     for (int k = 0; k < (int)fin.size(); ++k) {
       int old = raw_of[k];
       if (old < 0) continue;
-      std::set<int> ds;
-      for (int d : raw[r].deps[old]) ds.insert(remap(d));
+      std::set<int> ds, as;
+      auto add = [&](int d) { (is_ack(d) ? as : ds).insert(remap(d)); };
+      for (int d : raw[r].deps[old]) add(d);
       auto fr = fused_rev.find(old);
       if (fr != fused_rev.end())
-        for (int d : raw[r].deps[fr->second]) ds.insert(remap(d));
+        for (int d : raw[r].deps[fr->second]) add(d);
       ds.erase(k);
+      as.erase(k);
       fin[k].deps.assign(ds.begin(), ds.end());
+      fin[k].ack_deps.assign(as.begin(), as.end());
     }
     int ncta = std::max<int>({(int)RP.send_groups.size(), (int)RP.recv_groups.size(), 1});
     RP.ctas.assign(ncta, {});
@@ -347,20 +363,7 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
         std::stable_sort(l.begin(), l.end(), [&](int a, int b) { return fin[a].pc < fin[b].pc; });
         (lane == 0 ? RP.ctas[c].first : RP.ctas[c].second) = l;
       }
-    // direct mode: a dependency on a pull-send completes with the receiver's ack; it
-    // is never implied by lane order (the pull-send itself returns before the read)
-    if (P.direct) {
-      for (auto& p : fin) {
-        std::vector<int> keep;
-        for (int d : p.deps) {
-          if ((fin[d].flags & kDirect) && (fin[d].flags & kSend) && (fin[d].flags & kPull))
-            p.ack_deps.push_back(d);
-          else
-            keep.push_back(d);
-        }
-        p.deps = keep;
-      }
-    }
+    // (ack dependencies are never implied by lane order: a pull-send returns before the read)
     // drop dependencies implied by lane order
     std::map<int, std::tuple<int, int, int>> where;
     for (int c = 0; c < ncta; ++c) {
@@ -389,7 +392,6 @@ Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<i
   P.ir = ir;
   P.model = m;
   P.direct = direct;
-  if (direct) fuse = false;
   P.dag = build_dag(ir);
   P.pr = pr_in ? *pr_in : hpds(ir, P.dag, m);
   const int T = (int)ir.t.size(), N = ir.nranks;
@@ -454,12 +456,12 @@ Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<i
     rv.lane = 1;
     if (direct) {
       if (x.op == Op::Rrc) {  // pull: receiver reads the sender's location
-        s.flags |= kDirect | kPull;
+        s.flags |= kDirect | kSendPull;
         rv.flags |= kDirect | kPull;
         rv.rem_buf = s.src_buf;
       } else {                // push: sender writes the receiver's location
         s.flags |= kDirect;
-        s.rem_buf = rv.dst_buf;
+        s.rem_out = rv.dst_buf;
         rv.flags = kRecv | kDirect;
       }
       raw[x.src].prims[send_of[i].second] = s;
@@ -533,15 +535,40 @@ Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<i
   build_ranks(P, raw, any ? absorbed : none, loc_acc, written);
   P.fused = any;
   if (any) {
-    bool ok = true;
-    for (int nmb : {1, 2, 3, 16}) ok = ok && deadlock_free(P, 1, nmb);
-    if (!ok) {
+    auto check = [&]() {
+      bool ok = true;
+      for (int nmb : {1, 2, 3, 16}) ok = ok && deadlock_free(P, 1, nmb);
+      return ok;
+    };
+    auto rebuild = [&](const std::vector<std::map<int, int>>& ab) {
       for (auto& RP : P.ranks) {
         RP.prims.clear();
         RP.ctas.clear();
       }
-      build_ranks(P, raw, none, loc_acc, written);
-      P.fused = false;
+      build_ranks(P, raw, ab, loc_acc, written);
+    };
+    if (!check()) {
+      // direct mode: fusions whose send part only posts "readable" add no wait edge and
+      // are kept; push-forwarding fusions can form rendezvous cycles (R21/R23)
+      std::vector<std::map<int, int>> safe(N);
+      bool any_safe = false;
+      if (direct)
+        for (int r = 0; r < N; ++r)
+          for (auto& kv : absorbed[r])
+            if (raw[r].prims[kv.first].flags & kSendPull) {
+              safe[r][kv.first] = kv.second;
+              any_safe = true;
+            }
+      if (any_safe) {
+        rebuild(safe);
+        if (!check()) {
+          rebuild(none);
+          any_safe = false;
+        }
+      } else {
+        rebuild(none);
+      }
+      P.fused = any_safe;
     }
   }
   return P;
@@ -583,27 +610,26 @@ bool deadlock_free(const Plan& P, int K, int n_mb, std::string* why) {
     }
     return true;
   };
+  auto send_ok = [&](const Proc& p, const Prim& pm) {
+    if (!(pm.flags & kSend)) return true;
+    long pos = pos_of(pm.send_task, p.j);
+    if (!(pm.flags & kDirect)) return pos < credit[link(pm.send_task)] + K;
+    if (pm.flags & kSendPull) return true;                      // pull-send: post "readable"
+    return credit[link(pm.send_task)] >= pos + 1;               // push: receiver location writable
+  };
   auto enabled = [&](Proc& p) {
     if (p.k >= (int)p.prog->size()) return false;
     const Prim& pm = P.ranks[p.r].prims[(*p.prog)[p.k]];
     if (pm.flags & kCopy) return true;
     const bool direct = pm.flags & kDirect, pull = pm.flags & kPull;
-    if (direct && (pm.flags & kRecv) && !pull && p.phase == 1)  // push receiver waiting for payload
-      return produced[link(pm.recv_task)].count(pos_of(pm.recv_task, p.j)) > 0;
+    const bool push_recv = direct && (pm.flags & kRecv) && !pull;
+    if (push_recv && p.phase == 1)  // push receiver waiting for the payload (and its own send credit)
+      return produced[link(pm.recv_task)].count(pos_of(pm.recv_task, p.j)) > 0 && send_ok(p, pm);
     if (!deps_ok(p, pm)) return false;
-    if (pm.flags & kRecv) {
-      if (!direct || pull)
-        if (!produced[link(pm.recv_task)].count(pos_of(pm.recv_task, p.j))) return false;
-    }
-    if (pm.flags & kSend) {
-      long pos = pos_of(pm.send_task, p.j);
-      if (!direct) {
-        if (pos >= credit[link(pm.send_task)] + K) return false;
-      } else if (!pull) {
-        if (credit[link(pm.send_task)] < pos + 1) return false;
-      }
-    }
-    return true;
+    if (push_recv) return true;     // phase 0: post "writable"
+    if (pm.flags & kRecv)
+      if (!produced[link(pm.recv_task)].count(pos_of(pm.recv_task, p.j))) return false;
+    return send_ok(p, pm);
   };
   auto fire = [&](Proc& p) {
     int pid = (*p.prog)[p.k];
@@ -617,7 +643,7 @@ bool deadlock_free(const Plan& P, int K, int n_mb, std::string* why) {
     p.phase = 0;
     if (pm.recv_task >= 0) {
       long pos = pos_of(pm.recv_task, p.j);
-      if (!direct || pull) produced[link(pm.recv_task)].erase(pos);
+      produced[link(pm.recv_task)].erase(pos);
       if (!direct)
         credit[link(pm.recv_task)] += 1;
       else if (pull)
@@ -717,7 +743,7 @@ std::string plan_json(const Plan& P) {
         << ",\"recv_task\":" << p.recv_task << ",\"send_task\":" << p.send_task << ",\"src\":\""
         << buf_name(p.src_buf) << "\",\"dst\":\"" << buf_name(p.dst_buf) << "\",\"cta\":" << p.cta
         << ",\"lane\":" << p.lane << ",\"counter\":" << (p.has_counter ? "true" : "false")
-        << ",\"rem\":\"" << buf_name(p.rem_buf) << "\",\"deps\":[";
+        << ",\"rem\":\"" << buf_name(p.rem_buf) << "\",\"rem_out\":\"" << buf_name(p.rem_out) << "\",\"deps\":[";
       for (size_t d = 0; d < p.deps.size(); ++d) o << (d ? "," : "") << p.deps[d];
       o << "],\"ack_deps\":[";
       for (size_t d = 0; d < p.ack_deps.size(); ++d) o << (d ? "," : "") << p.ack_deps[d];

@@ -49,7 +49,8 @@ enum PrimFlags : int {
   // rrc tasks are pulled: the sender only posts "readable" and the receiver reads the
   // sender's location; the sender's completion is the receiver's read acknowledgement.
   kDirect = 32,
-  kPull = 64,    // with kDirect: payload read from the peer's buffer (rrc tasks)
+  kPull = 64,      // with kDirect + kRecv: the incoming payload is read from the peer (rrc task)
+  kSendPull = 128, // with kDirect + kSend: the outgoing task is pulled -- post "readable" only
 };
 
 struct Prim {
@@ -64,7 +65,8 @@ struct Prim {
   int lane = 0;         // 0 = send lane, 1 = recv lane
   std::vector<int> deps;  // prim ids on this rank whose same-micro-batch completion is awaited
   std::vector<int> ack_deps;  // direct mode: pull-send prims whose completion is the peer's ack
-  int rem_buf = BufNone;  // direct mode: buffer of the peer's location (push target / pull source)
+  int rem_buf = BufNone;  // direct mode: buffer of the peer location a pull reads
+  int rem_out = BufNone;  // direct mode: buffer of the peer location a push writes
   bool has_counter = false;
   const char* kind_name() const;
 };
