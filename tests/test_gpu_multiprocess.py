@@ -18,7 +18,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, algo, coll, count, dtype, q):
+def _worker(rank, world, port, algo, coll, count, dtype, q, opts="chunkbytes=4096 instances=2 fifodepth=2"):
     try:
         import sys
         root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -36,7 +36,7 @@ def _worker(rank, world, port, algo, coll, count, dtype, q):
         comm = R.init_process_group_comm(rank, world, 0)
         text = R.rescclGenerateIr(algo, coll, world)
         hdr, rest = text.split("\n", 1)
-        comm.load(hdr + " chunkbytes=4096 instances=2 fifodepth=2\n" + rest)
+        comm.load(hdr + " " + opts + "\n" + rest)
         m = count * world if coll == "reducescatter" else count
         x = inp.rank_input(dtype, 3, rank, m)
         s = to_torch(x, dtype)
@@ -87,6 +87,41 @@ def test_ipc_processes_match_oracle(algo, coll, world):
     m = count * world if coll == "reducescatter" else count
     xs = [inp.rank_input(dtype, 3, r, m) for r in range(world)]
     exp = replay.replay(lower.lower(g), xs, dtype, count, chunk_bytes=4096, instances=2, K=2)
+    for r in range(world):
+        outs, err = res[r]
+        assert err == 0
+        for o in outs:
+            assert np.array_equal(o.view(np.uint8), exp[r].view(np.uint8)), f"rank {r}"
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("algo,coll,world", [("ring", "allreduce", 2), ("ring", "allgather", 2)])
+def test_ipc_tma_engine_matches_oracle(algo, coll, world):
+    """Slices above tmamin: the TMA lane engine with .sys-scope flags across processes."""
+    import torch.multiprocessing as mp
+    import resccl_inputs as inp
+    from oracle import ir as oir, lower, replay
+    count, dtype = (6 << 20) + 33, "float32"
+    opts = "chunkbytes=4194304 instances=2 fifodepth=2"
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    os.environ["RESCCL_TIMEOUT_MS"] = "120000"
+    procs = [ctx.Process(target=_worker, args=(r, world, port, algo, coll, count, dtype, q, opts))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        rank, outs, err, tb = q.get(timeout=280)
+        assert tb is None, tb
+        res[rank] = (outs, err)
+    for p in procs:
+        p.join(30)
+    g = oir.generate(algo, coll, world)
+    m = count * world if coll == "reducescatter" else count
+    xs = [inp.rank_input(dtype, 3, r, m) for r in range(world)]
+    exp = replay.replay(lower.lower(g), xs, dtype, count, chunk_bytes=4194304, instances=2, K=2)
     for r in range(world):
         outs, err = res[r]
         assert err == 0
