@@ -97,6 +97,19 @@ rescclResult_t rescclCommConnect(rescclComm_t comm, const void* const* handles, 
 rescclResult_t rescclCommInit(rescclComm_t* out, int rank, int nranks, int cudaDev,
                               int (*allgather)(const void* in, void* out, size_t len, void* ctx), void* ctx);
 
+/* Symmetric windows for the direct transport across processes (reading R23):
+ * rescclCommRegister exports `bytes` of device memory at `ptr` (any pointer into a
+ * cudaMalloc'ed / caching-allocator block; the whole block is IPC-shared) as a blob
+ * (size protocol as rescclCommGetHandle); after the blobs are exchanged,
+ * rescclCommRegisterConnect maps every peer's window (blobs[k] = rank k's blob) and
+ * returns its id.  Every rank registers its corresponding buffer in the same order
+ * with the same size.  An algorithm loaded with direct=1 then runs its direct kernel
+ * when a call's send and receive buffers lie in registered windows at the same
+ * offsets on every rank, and its staged twin otherwise (and for ReduceScatter). */
+rescclResult_t rescclCommRegister(rescclComm_t comm, void* ptr, size_t bytes, void* blob, size_t* len);
+rescclResult_t rescclCommRegisterConnect(rescclComm_t comm, const void* const* blobs, const size_t* lens,
+                                         int* window);
+
 /* Single-process communicators: comms[k] is rank k on device devlist[k].  Repeated
  * devices host virtual ranks (see "Execution modes").  devlist == NULL means all
  * ranks on device 0. */

@@ -46,6 +46,7 @@ EXPORTS = [
     "rescclAllReduce",
     "rescclAllGather", "rescclReduceScatter", "rescclGenerateIr", "rescclPlanIr",
     "rescclCodegenIr", "rescclCompileIr", "rescclCheckDeadlock", "rescclParseResCCLang", "rescclProfilePlanner",
+    "rescclCommRegister", "rescclCommRegisterConnect",
 ]
 
 _c = ctypes
@@ -76,6 +77,8 @@ _SIGS = {
     "rescclCheckDeadlock": (_i, [_c.c_char_p, _c.c_char_p, _i, _i, _c.POINTER(_i)]),
     "rescclParseResCCLang": (_i, [_c.c_char_p, _c.c_char_p, _c.POINTER(_sz)]),
     "rescclProfilePlanner": (_i, [_c.c_char_p, _c.c_char_p, _i, _c.c_char_p, _c.POINTER(_sz)]),
+    "rescclCommRegister": (_i, [_vp, _vp, _sz, _vp, _c.POINTER(_sz)]),
+    "rescclCommRegisterConnect": (_i, [_vp, _c.POINTER(_vp), _c.POINTER(_sz), _c.POINTER(_i)]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -155,6 +158,23 @@ def rescclCommInitAll(devices: Sequence[int]) -> List[int]:
     devs = (_i * n)(*devices)
     _check(_lib.rescclCommInitAll(comms, n, devs), "rescclCommInitAll")
     return [comms[k] for k in range(n)]
+
+
+def rescclCommRegister(comm: int, ptr: int, nbytes: int) -> bytes:
+    n = _sz(0)
+    _check(_lib.rescclCommRegister(comm, ptr, nbytes, None, _c.byref(n)), "rescclCommRegister")
+    buf = _c.create_string_buffer(n.value)
+    _check(_lib.rescclCommRegister(comm, ptr, nbytes, _c.cast(buf, _vp), _c.byref(n)), "rescclCommRegister")
+    return buf.raw[:n.value]
+
+
+def rescclCommRegisterConnect(comm: int, blobs: Sequence[bytes]) -> int:
+    bufs = [_c.create_string_buffer(h, len(h)) for h in blobs]
+    arr = (_vp * len(bufs))(*[_c.cast(b, _vp) for b in bufs])
+    lens = (_sz * len(bufs))(*[len(h) for h in blobs])
+    w = _i()
+    _check(_lib.rescclCommRegisterConnect(comm, arr, lens, _c.byref(w)), "rescclCommRegisterConnect")
+    return w.value
 
 
 def rescclCommDestroy(comm: int) -> None:

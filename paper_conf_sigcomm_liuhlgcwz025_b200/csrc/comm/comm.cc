@@ -51,6 +51,7 @@ struct KArgs {
   int* err;
   unsigned long long timeout_ns;
   unsigned long long* trace;
+  unsigned long long epoch;
 };
 
 thread_local std::string g_last_error;
@@ -77,6 +78,7 @@ struct Driver {
                            CUstream, void**, void**) = nullptr;
   CUresult (*GetErrorString)(CUresult, const char**) = nullptr;
   CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
+  CUresult (*MemGetAddressRange)(CUdeviceptr*, size_t*, CUdeviceptr) = nullptr;
   bool ok = false;
 };
 
@@ -101,6 +103,7 @@ Driver& driver() {
       entry("cuLaunchKernel", &d.LaunchKernel);
       entry("cuGetErrorString", &d.GetErrorString);
       entry("cuFuncSetAttribute", &d.FuncSetAttribute);
+      entry("cuMemGetAddressRange", &d.MemGetAddressRange);
       d.ok = true;
     } catch (Error&) {
       d.ok = false;
@@ -138,6 +141,7 @@ struct Options {
   int backoff = 1;
   int jitter = 0;
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
+  int sys_rank = -1; // rescclCompileIr / rescclCodegenIr: one rank's multi-process (.sys) kernel
 };
 
 std::map<std::string, std::string> parse_kv(const char* s) {
@@ -181,6 +185,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "direct") o.direct = (int)to_long(v, k);
   else if (k == "backoff") o.backoff = (int)to_long(v, k);
   else if (k == "jitter") o.jitter = (int)to_long(v, k);
+  else if (k == "sysrank") o.sys_rank = (int)to_long(v, k);
   else if (k == "sched") {
     if (v == "hpds") o.sched = 0;
     else if (v == "rr") o.sched = 1;
@@ -323,6 +328,7 @@ struct AlgoShared {
   unsigned long long* trace_dev = nullptr;
   int trace_blocks = 0;                // blocks covered by the last traced launch
   int trace_block_base = 0;
+  std::shared_ptr<AlgoShared> twin;    // multi-process direct plan: staged plan for unregistered buffers
   char* region_alloc = nullptr;
   int64_t region_off = 0;              // multi-process: offset inside the arena
 };
@@ -332,7 +338,9 @@ struct AlgoShared {
 struct rescclAlgo {
   std::shared_ptr<AlgoShared> s;
   rescclComm* comm = nullptr;
-  unsigned long long mb_cum = 0;  // multi-process: this rank's counter
+  unsigned long long mb_cum = 0;       // multi-process: this rank's counter
+  unsigned long long twin_mb_cum = 0;  // ... and its staged twin's
+  unsigned long long epoch = 0;        // direct calls issued (exit-barrier target)
 };
 
 namespace {
@@ -355,6 +363,15 @@ struct rescclComm {
   char* scratch = nullptr;
   size_t scratch_bytes = 0;
   std::vector<rescclComm*> peers_local;  // mode 2: every comm of the process
+  // registered symmetric windows (multi-process direct transport): local range and every
+  // peer's corresponding range as mapped in this process
+  struct Window {
+    char* base = nullptr;
+    size_t bytes = 0;
+    std::vector<char*> peer;
+  };
+  std::vector<Window> windows;
+  std::map<std::string, char*> ipc_maps;  // opened peer allocations (handle bytes -> mapped base)
 };
 
 namespace {
@@ -408,7 +425,7 @@ Ir parse_any(const std::string& text) {
   return parse_ir(text);
 }
 
-std::shared_ptr<AlgoShared> build_algo(const std::string& text, int nranks) {
+std::shared_ptr<AlgoShared> build_algo(const std::string& text, int nranks, const char* extra = nullptr) {
   auto a = std::make_shared<AlgoShared>();
   a->text = text;
   try {
@@ -421,7 +438,7 @@ std::shared_ptr<AlgoShared> build_algo(const std::string& text, int nranks) {
                                  std::to_string(nranks));
   if (nranks > kMaxR) fail(rescclInvalidUsage, "at most 32 ranks per communicator");
   try {
-    a->opt = make_options(a->ir, nullptr);
+    a->opt = make_options(a->ir, extra);
     a->plan = plan_checked(a->ir, a->opt);
     a->lay = make_layout(a->plan, a->opt.fifo_depth, a->opt.instances, a->opt.chunk_bytes);
   } catch (PlanError& e) {
@@ -469,6 +486,7 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.tma_min = a.opt.tma_min;
   co.backoff = a.opt.backoff;
   co.jitter = a.opt.jitter;
+  co.exit_barrier = a.opt.direct && !gpu_scope;
   std::string src = codegen(a.plan, a.lay, co);
   if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
     if (FILE* f = fopen((std::string(dump) + "_" + a.ir.name + "_" + coll_name(a.ir.coll) + ".cu").c_str(), "w")) {
@@ -585,10 +603,39 @@ unsigned long long* trace_buffer(AlgoShared& a, int blocks, int block_base) {
   return a.trace_dev;
 }
 
+// connected window containing [p, p + bytes), or -1
+int find_window(const rescclComm* comm, const void* p, size_t bytes) {
+  for (size_t w = 0; w < comm->windows.size(); ++w) {
+    const auto& W = comm->windows[w];
+    bool connected = true;
+    for (char* q : W.peer) connected = connected && q;
+    if (connected && (const char*)p >= W.base && (const char*)p + bytes <= W.base + W.bytes) return (int)w;
+  }
+  return -1;
+}
+
 // multi-process / multi-device path: this rank alone
+
 void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const void* send, void* recv,
                  cudaStream_t s) {
-  AlgoShared& a = *algo->s;
+  AlgoShared* ap = algo->s.get();
+  unsigned long long* mb_cum = &algo->mb_cum;
+  int ws = -1, wr = -1;
+  if (ap->opt.direct && comm->mode == 0) {
+    // direct transport across processes needs both buffers in registered symmetric
+    // windows (same window and offset on every rank); otherwise the staged twin runs
+    const size_t e = elt_size(c.dt);
+    const size_t sb = c.count * e * (c.coll == (int)Coll::ReduceScatter ? comm->nranks : 1);
+    const size_t rb = c.count * e * (c.coll == (int)Coll::AllGather ? comm->nranks : 1);
+    ws = find_window(comm, send, sb);
+    wr = find_window(comm, recv, rb);
+    if (ws < 0 || wr < 0 || c.coll == (int)Coll::ReduceScatter) {
+      ap = ap->twin.get();
+      mb_cum = &algo->twin_mb_cum;
+      ws = wr = -1;
+    }
+  }
+  AlgoShared& a = *ap;
   Geometry g = call_geometry(a, c);
   if (g.n_mb == 0) return;
   cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
@@ -597,12 +644,22 @@ void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const vo
   for (int q = 0; q < comm->nranks; ++q) ka.arena[q] = comm->peer_arena[q] + a.region_off;
   ka.sendbuf[comm->rank] = (const char*)send;
   ka.recvbuf[comm->rank] = (char*)recv;
+  if (ws >= 0) {
+    const auto& WS = comm->windows[ws];
+    const auto& WR = comm->windows[wr];
+    const size_t os = (const char*)send - WS.base, orr = (char*)recv - WR.base;
+    for (int q = 0; q < comm->nranks; ++q) {
+      ka.sendbuf[q] = WS.peer[q] + os;
+      ka.recvbuf[q] = WR.peer[q] + orr;
+    }
+  }
   if (a.ir.coll == Coll::ReduceScatter) {
     ensure_scratch(comm, c.count * comm->nranks * elt_size(c.dt));
     ka.scratch[comm->rank] = comm->scratch;
   }
   fill_geometry(ka, g, c.count);
-  ka.mb_base = algo->mb_cum;
+  ka.mb_base = *mb_cum;
+  if (ws >= 0) ka.epoch = algo->epoch++;
   ka.block_base = a.lay.pair_start[comm->rank] * a.opt.instances;
   ka.err = comm->err_dev;
   ka.timeout_ns = timeout_ns();
@@ -610,7 +667,7 @@ void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const vo
   const bool use_tma = a.opt.tma && g.Mi * elt_size(c.dt) >= a.opt.tma_min;
   Kern& k = get_kernel(a, c.dt, c.op, comm->rank, comm->rank + 1, false, use_tma);
   launch(k, a.lay.ctas[comm->rank] * a.opt.instances, 32 * a.opt.nwarps, ka, s);
-  algo->mb_cum += (unsigned long long)g.n_mb;
+  *mb_cum += (unsigned long long)g.n_mb;
 }
 
 // virtual group: all ranks in one kernel, when the last rank arrives
@@ -728,15 +785,20 @@ rescclAlgo* load_algo(rescclComm* comm, const std::string& text) {
     }
   } else {
     s = build_algo(text, comm->nranks);
-    if (s->opt.direct)
-      fail(rescclInvalidUsage, "direct=1 needs every rank's buffers in one address space (virtual ranks); "
-                               "multi-process communicators use the staged FIFO transport");
-    size_t need = (size_t)s->lay.region_bytes;
-    if (comm->arena_used + need > comm->arena_bytes)
-      fail(rescclInvalidUsage, "FIFO arena exhausted: need " + std::to_string(comm->arena_used + need) +
-                                   " bytes; raise RESCCL_ARENA_BYTES");
-    s->region_off = (int64_t)comm->arena_used;
-    comm->arena_used += (need + 4095) / 4096 * 4096;
+    if (s->opt.direct) {
+      if (comm->mode != 0)
+        fail(rescclInvalidUsage, "direct=1 is supported for virtual ranks and multi-process communicators");
+      s->twin = build_algo(text, comm->nranks, "direct=0");  // staged plan for unregistered buffers
+    }
+    for (AlgoShared* x : {s.get(), s->twin.get()}) {
+      if (!x) continue;
+      size_t need = (size_t)x->lay.region_bytes;
+      if (comm->arena_used + need > comm->arena_bytes)
+        fail(rescclInvalidUsage, "FIFO arena exhausted: need " + std::to_string(comm->arena_used + need) +
+                                     " bytes; raise RESCCL_ARENA_BYTES");
+      x->region_off = (int64_t)comm->arena_used;
+      comm->arena_used += (need + 4095) / 4096 * 4096;
+    }
   }
   auto algo = std::make_unique<rescclAlgo>();
   algo->s = s;
@@ -873,6 +935,81 @@ rescclResult_t rescclCommConnect(rescclComm_t comm, const void* const* handles, 
   API_END
 }
 
+struct WinBlob {
+  unsigned magic;
+  int rank;
+  unsigned long long bytes, offset;
+  cudaIpcMemHandle_t handle;
+};
+
+rescclResult_t rescclCommRegister(rescclComm_t comm, void* ptr, size_t bytes, void* blob, size_t* len) {
+  API_BEGIN
+  if (!comm || !len) fail(rescclInvalidArgument, "null argument");
+  if (comm->mode != 0) fail(rescclInvalidUsage, "windows are for multi-process communicators");
+  if (!blob) {
+    *len = sizeof(WinBlob);
+    return rescclSuccess;
+  }
+  if (!ptr || bytes == 0) fail(rescclInvalidArgument, "null or empty window");
+  if (*len < sizeof(WinBlob)) fail(rescclInvalidArgument, "blob buffer too small");
+  cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+  CUdeviceptr base = 0;
+  size_t asz = 0;
+  cu_check(driver().MemGetAddressRange(&base, &asz, (CUdeviceptr)ptr), "cuMemGetAddressRange");
+  if ((char*)ptr + bytes > (char*)base + asz) fail(rescclInvalidArgument, "window exceeds its allocation");
+  WinBlob b;
+  memset(&b, 0, sizeof(b));
+  b.magic = 0x52574e44u;
+  b.rank = comm->rank;
+  b.bytes = bytes;
+  b.offset = (char*)ptr - (char*)base;
+  cuda_check(cudaIpcGetMemHandle(&b.handle, (void*)base), "cudaIpcGetMemHandle(window)");
+  memcpy(blob, &b, sizeof(b));
+  *len = sizeof(b);
+  rescclComm::Window W;
+  W.base = (char*)ptr;
+  W.bytes = bytes;
+  W.peer.assign(comm->nranks, nullptr);
+  W.peer[comm->rank] = (char*)ptr;
+  comm->windows.push_back(W);  // connected by rescclCommRegisterConnect
+  API_END
+}
+
+rescclResult_t rescclCommRegisterConnect(rescclComm_t comm, const void* const* blobs, const size_t* lens,
+                                         int* window) {
+  API_BEGIN
+  if (!comm || !blobs || !lens) fail(rescclInvalidArgument, "null argument");
+  if (comm->windows.empty()) fail(rescclInvalidUsage, "rescclCommRegister first");
+  auto& W = comm->windows.back();
+  cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+  for (int q = 0; q < comm->nranks; ++q) {
+    if (q == comm->rank) continue;
+    if (!blobs[q] || lens[q] < sizeof(WinBlob)) fail(rescclInvalidArgument, "bad window blob");
+    WinBlob b;
+    memcpy(&b, blobs[q], sizeof(b));
+    if (b.magic != 0x52574e44u || b.rank != q) fail(rescclInvalidArgument, "inconsistent window blob");
+    if (b.bytes != W.bytes) fail(rescclInvalidUsage, "windows must have the same size on every rank");
+    std::string key(reinterpret_cast<const char*>(&b.handle), sizeof(b.handle));
+    key += "/" + std::to_string(q);
+    auto it = comm->ipc_maps.find(key);
+    char* mapped;
+    if (it != comm->ipc_maps.end()) {
+      mapped = it->second;
+    } else {
+      void* p = nullptr;
+      cudaError_t e = cudaIpcOpenMemHandle(&p, b.handle, cudaIpcMemLazyEnablePeerAccess);
+      if (e != cudaSuccess)
+        fail(rescclSystemError, "cudaIpcOpenMemHandle(window of rank " + std::to_string(q) + "): " +
+                                    cudaGetErrorString(e));
+      mapped = (char*)p;
+      comm->ipc_maps[key] = mapped;
+    }
+    W.peer[q] = mapped + b.offset;
+  }
+  if (window) *window = (int)comm->windows.size() - 1;
+  API_END
+}
+
 rescclResult_t rescclCommInit(rescclComm_t* out, int rank, int nranks, int cudaDev,
                               int (*allgather)(const void*, void*, size_t, void*), void* ctx) {
   API_BEGIN
@@ -992,11 +1129,14 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
   } else {
     for (auto& a : comm->algos) {
       if (a->s.use_count() == 1)
-        for (auto& k : a->s->kernels)
-          if (k.second.mod) driver().ModuleUnload(k.second.mod);
+        for (AlgoShared* x : {a->s.get(), a->s->twin.get()})
+          if (x)
+            for (auto& k : x->kernels)
+              if (k.second.mod) driver().ModuleUnload(k.second.mod);
     }
     for (int q = 0; q < (int)comm->peer_opened.size(); ++q)
       if (comm->peer_opened[q]) cudaIpcCloseMemHandle(comm->peer_arena[q]);
+    for (auto& kv : comm->ipc_maps) cudaIpcCloseMemHandle(kv.second);
     if (comm->arena) cudaFree(comm->arena);
     if (comm->err_host) cudaFreeHost(comm->err_host);
     if (comm->scratch) cudaFree(comm->scratch);
@@ -1227,7 +1367,14 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
   co.backoff = o.backoff;
   co.jitter = o.jitter;
   co.gpu_scope = true;
-  auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, true);
+  if (o.sys_rank >= 0) {  // one rank of a multi-process communicator
+    if (o.sys_rank >= p.ir.nranks) fail(rescclInvalidArgument, "sysrank out of range");
+    co.rank_lo = o.sys_rank;
+    co.rank_hi = o.sys_rank + 1;
+    co.gpu_scope = false;
+    co.exit_barrier = o.direct;
+  }
+  auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, co.gpu_scope);
   if (cubin_bytes) *cubin_bytes = cub.size();
   API_END
 }

@@ -56,6 +56,7 @@ struct KArgs {
   int* err;                           // host-mapped error word
   u64 timeout_ns;
   u64* trace;                         // RESCCL_TRACE: 4 x u64 per (block, lane), host-mapped
+  u64 epoch;                          // RESCCL_EXIT_BARRIER: calls of this plan issued before
 };
 
 enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16, kDirect = 32, kPull = 64, kSendPull = 128 };
@@ -991,6 +992,32 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
   }
 #endif
   return run_sync<T, OP, F>(L, d, p);
+}
+
+// Direct transport across processes (RESCCL_EXIT_BARRIER): peers pull from and push into
+// this rank's user buffers, so this rank's kernel -- whose completion hands the buffers
+// back to the caller -- must not end before every peer block is done with them.  Every
+// block adds 1 to its rank's monotone done counter (release); block 0 then waits until
+// each peer's counter covers this call: (epoch + 1) x that peer's block count.
+__device__ __noinline__ void exit_barrier(const KArgs& a, int rank, int nranks, const int* blocks, i64 off) {
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  fence_release();
+  asm volatile("red.release" RESCCL_SC ".global.add.u64 [%0], 1;" ::"l"(at(a.arena[rank], off)) : "memory");
+  if (blockIdx.x != 0) return;
+  const u64 t0 = globaltimer();
+  for (int q = 0; q < nranks; ++q) {
+    if (q == rank) continue;
+    const u64 target = (a.epoch + 1) * (u64)blocks[q];
+    u32 spins = 0;
+    while (ld_acquire(at(a.arena[q], off)) < target) {
+      if (++spins > 64) nanosleep_(64);
+      if ((spins & 1023) == 0 && globaltimer() - t0 > a.timeout_ns) {
+        atomicCAS(a.err, 0, kErrTimeout);
+        return;
+      }
+    }
+  }
 }
 
 }  // namespace rdev

@@ -29,6 +29,7 @@ struct Layout {
   std::vector<std::vector<int>> ctr_slot;              // prim -> counter slot (-1: none)
   std::vector<int64_t> cred_base, ctr_base, flag_base, data_base, bytes;
   int64_t region_bytes = 0;  // max over ranks (regions sit at the same arena offset)
+  int64_t done_off = 0;      // exit-barrier counter (direct transport across processes)
   // TB geometry
   std::vector<int> ctas;        // per rank
   std::vector<int> pair_start;  // per rank: index of (rank, cta 0) among all (rank, cta) pairs
@@ -50,6 +51,8 @@ struct CodegenOpts {
   int backoff = 1;               // nanosleep back-off while polling flags
   int jitter = 0;                // debug fault injector: random delays around every sync
   int prefetch = 0;              // micro-batches of local operand prefetched into L2 ahead (off: r01)
+  int exit_barrier = 0;          // direct transport across processes: a rank's kernel ends only
+                                 // after every peer's blocks finished touching its buffers
 };
 
 // dynamic shared memory the generated kernel needs (both lanes' TMA staging)

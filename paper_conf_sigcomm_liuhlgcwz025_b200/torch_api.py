@@ -59,6 +59,15 @@ class Communicator:
     def async_error(self) -> int:
         return _r.rescclCommGetAsyncError(self.handle)
 
+    def register(self, tensor, group=None) -> int:
+        """Register `tensor` as a symmetric window (collective over the process group):
+        export, exchange the blobs with all_gather_object, map the peers' windows."""
+        import torch.distributed as dist
+        blob = _r.rescclCommRegister(self.handle, tensor.data_ptr(), tensor.numel() * tensor.element_size())
+        blobs: List[Optional[bytes]] = [None] * self.nranks
+        dist.all_gather_object(blobs, blob, group=group)
+        return _r.rescclCommRegisterConnect(self.handle, blobs)
+
     def destroy(self):
         if self.handle:
             _r.rescclCommDestroy(self.handle)

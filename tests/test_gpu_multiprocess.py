@@ -127,3 +127,94 @@ def test_ipc_tma_engine_matches_oracle(algo, coll, world):
         assert err == 0
         for o in outs:
             assert np.array_equal(o.view(np.uint8), exp[r].view(np.uint8)), f"rank {r}"
+
+
+def _window_worker(rank, world, port, algo, coll, count, dtype, q, opts):
+    """Direct transport across processes: buffers registered as symmetric windows run
+    the direct kernel; an unregistered buffer runs the staged twin (reading R23)."""
+    try:
+        import sys
+        root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+        sys.path.insert(0, root)
+        sys.path.insert(0, os.path.join(root, "tests"))
+        import torch
+        import torch.distributed as dist
+        import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+        import resccl_inputs as inp
+        from gpu_helpers import to_numpy, to_torch, poison
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        comm = R.init_process_group_comm(rank, world, 0)
+        text = R.rescclGenerateIr(algo, coll, world)
+        hdr, rest = text.split("\n", 1)
+        comm.load(hdr + " " + opts + "\n" + rest)
+        m = count * world if coll == "reducescatter" else count
+        n_out = count * world if coll == "allgather" else count
+        x = to_torch(inp.rank_input(dtype, 3, rank, m), dtype)
+        # one window holding send and receive buffers at symmetric offsets
+        win = torch.empty(m + n_out + 64, dtype=x.dtype, device="cuda:0")
+        comm.register(win)
+        s_reg, r_reg = win[:m], win[m + 64:m + 64 + n_out]
+        s_reg.copy_(x)
+        outs = []
+        for it, reg in enumerate([True, False, True, True]):
+            s = s_reg if reg else x
+            r = r_reg if reg else torch.empty(n_out, dtype=x.dtype, device="cuda:0")
+            poison(r)
+            torch.cuda.synchronize()
+            dist.barrier()
+            getattr(comm, coll)(s, r)
+            torch.cuda.synchronize()
+            outs.append(to_numpy(r.clone(), dtype))
+        err = comm.async_error()
+        dist.barrier()
+        comm.destroy()
+        dist.destroy_process_group()
+        q.put((rank, outs, err, None))
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put((rank, None, None, traceback.format_exc()))
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("algo,coll,world,count,opts", [
+    ("ring", "allreduce", 2, 9000, "chunkbytes=4096 instances=2 fifodepth=2 direct=1"),
+    ("ring", "allgather", 2, 9000, "chunkbytes=4096 instances=2 fifodepth=2 direct=1"),
+    ("ring", "reducescatter", 2, 9000, "chunkbytes=4096 instances=2 fifodepth=2 direct=1"),
+    ("dbt", "allreduce", 4, 9000, "chunkbytes=4096 instances=2 fifodepth=2 direct=1"),
+    ("ring", "allreduce", 2, (6 << 20) + 33, "chunkbytes=4194304 instances=2 fifodepth=2 direct=1"),
+])
+def test_ipc_registered_windows_direct(algo, coll, world, count, opts):
+    import torch.multiprocessing as mp
+    import resccl_inputs as inp
+    from oracle import ir as oir, lower, replay
+    dtype = "float32"
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    os.environ["RESCCL_TIMEOUT_MS"] = "120000"
+    procs = [ctx.Process(target=_window_worker, args=(r, world, port, algo, coll, count, dtype, q, opts))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        rank, outs, err, tb = q.get(timeout=280)
+        assert tb is None, tb
+        res[rank] = (outs, err)
+    for p in procs:
+        p.join(30)
+    g = oir.generate(algo, coll, world)
+    m = count * world if coll == "reducescatter" else count
+    xs = [inp.rank_input(dtype, 3, r, m) for r in range(world)]
+    cb = int(opts.split("chunkbytes=")[1].split()[0])
+    exp_d = replay.replay(lower.lower(g, direct=True), xs, dtype, count, chunk_bytes=cb, instances=2, K=2)
+    exp_s = replay.replay(lower.lower(g), xs, dtype, count, chunk_bytes=cb, instances=2, K=2)
+    for r in range(world):
+        outs, err = res[r]
+        assert err == 0
+        for it, o in enumerate(outs):
+            e = exp_s if (it == 1 or coll == "reducescatter") else exp_d
+            assert np.array_equal(o.view(np.uint8), e[r].view(np.uint8)), f"rank {r} call {it}"

@@ -193,6 +193,16 @@ def test_generated_kernel_compiles_for_sm100a(name, coll, n, kw, dtype):
     assert R.rescclCompileIr(text, "instances=2", dtype, R.rescclSum) > 10000
 
 
+@pytest.mark.parametrize("direct", [0, 1])
+def test_multiprocess_rank_kernel_compiles(direct):
+    """One rank's multi-process kernel (.sys scope); with direct=1 it carries the exit
+    barrier that keeps peers' pulls/pushes inside the call (registered windows)."""
+    text = _cpp_ir("ring", "allreduce", 4, {})
+    assert R.rescclCompileIr(text, f"instances=2 sysrank=1 direct={direct}", R.rescclBfloat16, R.rescclSum) > 10000
+    src = R.rescclCodegenIr(text, f"direct={direct}", 1, 2)
+    assert "#define RESCCL_EXIT_BARRIER 0" in src  # CodegenIr leaves it to the runtime
+
+
 def test_generated_code_has_no_interpreter():
     """§4.5: every primitive is a direct call with compile-time descriptor; no loop over
     a runtime program array."""

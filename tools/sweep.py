@@ -81,18 +81,19 @@ if "c3" in which:
     for name, g in (("dbt", ""), ("hm", "g=4")):
         for budget in (1, 2, 4, 8, 12, 16):
             for S in (64 << 20, 256 << 20):
-                emit(measure(name, "allreduce", g, dict(chunkbytes=1 << 20, fifodepth=2, tbbudget=budget), S))
+                emit(measure(name, "allreduce", g, dict(chunkbytes=1 << 20, fifodepth=2, tbbudget=budget, direct=BASE["direct"]), S))
     for S in (64 << 20, 256 << 20):
-        emit(measure("ring", "allreduce", "", dict(chunkbytes=1 << 20, fifodepth=2, instances=2), S))
+        emit(measure("ring", "allreduce", "", dict(chunkbytes=1 << 20, fifodepth=2, instances=2,
+                                                   direct=BASE["direct"]), S))
 if "c4" in which:
     for coll in ("allgather", "reducescatter"):
         for fan in (2, 3):
             for S in (4 << 20, 16 << 20, 64 << 20, 256 << 20):
                 emit(measure("synth", coll, f"seed=0 fanout={fan}", dict(instances=4, chunkbytes=1 << 20,
-                                                                          fifodepth=2), S))
+                                                                          fifodepth=2, direct=BASE["direct"]), S))
 if "f2" in which:
     for name, coll, g in (("hm", "allreduce", "g=4"), ("hm", "allgather", "g=4"), ("dbt", "allreduce", ""),
                           ("synth", "allgather", "seed=0 fanout=2"), ("synth", "reducescatter", "seed=1 fanout=3")):
         for sched in ("hpds", "rr"):
-            emit(measure(name, coll, g, dict(instances=4, chunkbytes=1 << 20, fifodepth=2, sched=sched),
-                         64 << 20))
+            emit(measure(name, coll, g, dict(instances=4, chunkbytes=1 << 20, fifodepth=2, sched=sched,
+                                             direct=BASE["direct"]), 64 << 20))
