@@ -139,8 +139,22 @@ class _Sim:
     (``fifo``) and a monotone ``credit``: the receiver's consumption (staged), its
     "writable" posts (direct push) or its read acknowledgements (direct pull)."""
 
-    def __init__(self, plan: Plan, n_mb: int, instances: int, K: int):
+    def __init__(self, plan: Plan, n_mb: int, instances: int, K: int, rings: Optional[str] = None):
         self.plan, self.n_mb, self.I, self.K = plan, n_mb, instances, K
+        # Device-faithful flag model (R26): each payload flag lives in slot pos % K of a
+        # ring, overwritten with pos + 1 on every post; the receiver of pos tests
+        # "slot >= pos + 1".  rings="link": one ring per (link, instance); rings="lane":
+        # one ring per (link, instance, sending lane).  Every test of the device
+        # condition that disagrees with the ideal "pos was posted and not consumed"
+        # is recorded in self.hazards.
+        self.rings = rings
+        self.slots = defaultdict(dict)
+        self.hazards = []
+        self.send_lane = {}
+        for r, prims in plan.prims.items():
+            for pid, p in enumerate(prims):
+                if p.send_task is not None:
+                    self.send_lane[p.send_task] = (p.cta, p.lane)
         self.tasks = plan.ir.transfers
         order = conn_positions(plan)
         self.tpos = {}
@@ -187,6 +201,19 @@ class _Sim:
             return True
         return cr >= pos + 1                          # push: receiver location writable
 
+    def _ring(self, task, inst):
+        key = (self._link(task), inst)
+        return key + (self.send_lane[task],) if self.rings == "lane" else key
+
+    def _arrived(self, task, j, inst) -> bool:
+        pos = self.pos(task, j)
+        ideal = pos in self.fifo[(self._link(task), inst)]
+        if self.rings:
+            dev = self.slots[self._ring(task, inst)].get(pos % self.K, 0) >= pos + 1
+            if dev != ideal:
+                self.hazards.append((self._link(task), inst, pos, "early" if dev else "lost"))
+        return ideal
+
     def enabled(self, pr) -> bool:
         r, c, lane, inst, prog, k, j, phase = pr
         if k >= len(prog):
@@ -195,14 +222,13 @@ class _Sim:
         if p.kind == "copy":
             return True
         if p.kind in PUSH_RECVS and phase == 1:       # push receiver waiting for the payload
-            return (self.pos(p.recv_task, j) in self.fifo[(self._link(p.recv_task), inst)]
-                    and self.send_ok(p, j, inst))
+            return self._arrived(p.recv_task, j, inst) and self.send_ok(p, j, inst)
         if not self.deps_ok(r, p, j, inst):
             return False
         if p.kind in PUSH_RECVS:                      # phase 0: post "writable"
             return True
         if p.recv_task is not None:
-            if self.pos(p.recv_task, j) not in self.fifo[(self._link(p.recv_task), inst)]:
+            if not self._arrived(p.recv_task, j, inst):
                 return False
         return self.send_ok(p, j, inst)
 
@@ -233,6 +259,9 @@ class _Sim:
         if p.send_task is not None:
             key = (self._link(p.send_task), inst)
             self.fifo[key][self.pos(p.send_task, j)] = out
+            if self.rings:
+                pos = self.pos(p.send_task, j)
+                self.slots[self._ring(p.send_task, inst)][pos % self.K] = pos + 1
         if p.kind != "copy":
             self.done[(r, prog[k], inst)] = j + 1
         j += 1

@@ -28,6 +28,12 @@ struct Layout {
   std::vector<std::map<int, int>> send_idx, recv_idx;  // peer -> connection index
   std::vector<std::vector<int>> ctr_slot;              // prim -> counter slot (-1: none)
   std::vector<int64_t> cred_base, ctr_base, flag_base, data_base, bytes;
+  // Flag rings: one per (receive connection, sending lane).  A link whose sends come
+  // from several lanes (fused forwards beside plain sends) gets one ring per lane, so
+  // each ring is posted in increasing position order and "flag >= pos + 1" implies that
+  // pos was posted (R26).  task_sub[t] = ring of task t within its connection.
+  std::vector<std::vector<int>> flag_conn;  // per rank: first ring of each receive connection
+  std::vector<int> task_sub;
   int64_t region_bytes = 0;  // max over ranks (regions sit at the same arena offset)
   int64_t done_off = 0;      // exit-barrier counter (direct transport across processes)
   // TB geometry

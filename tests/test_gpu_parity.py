@@ -231,3 +231,22 @@ def test_direct_edge_counts_inplace(coll, count):
         assert err == 0
         exp = oracle_expect(g, xs, "bfloat16", count, chunk_bytes=65536, instances=3)
         _check_bytes(outs, exp, coll, n, count)
+
+
+@pytest.mark.parametrize("name,coll,kw,fifo", [("synth", "reducescatter", {"seed": 0, "fanout": 2}, 2),
+                                               ("synth", "reducescatter", {"seed": 0, "fanout": 2}, 1),
+                                               ("synth", "reducescatter", {"seed": 1, "fanout": 2}, 2),
+                                               ("ring", "allreduce", {}, 1),
+                                               ("synth", "allgather", {"seed": 0, "fanout": 3}, 1)])
+def test_direct_flag_rings_regression(name, coll, kw, fifo):
+    """R26 regression: links fed by two sending lanes under the direct transport, several
+    micro-batches, shallow flag rings (this hung before rings were split per lane)."""
+    n = 8
+    g = oir.generate(name, coll, n, **kw)
+    count = 5 * 2048 + 13
+    text = _hdr(g, chunkbytes=8192, instances=2, fifodepth=fifo, direct=1)
+    xs = _inputs(coll, "float32", n, count, seed=5)
+    outs, info, err = run_virtual(R, text, coll, xs, "float32", count)
+    assert err == 0 and info["direct"] == 1
+    exp = oracle_expect(g, xs, "float32", count, chunk_bytes=8192, instances=2, K=fifo)
+    _check_bytes(outs, exp, coll, n, count)

@@ -569,3 +569,34 @@ def test_direct_race_checker_catches_missing_ack_dependency():
         for p in pd.prims[r]:
             p.ack_deps = []
     assert replay.happens_before_races(pd, n_mb=2, instances=1, K=1, inplace=True) != []
+
+
+# ----------------------------------------------------------------------------- flag rings (R26)
+
+@pytest.mark.parametrize("name,coll,n,kw", [("ring", "allreduce", 8, {}),
+                                            ("synth", "reducescatter", 8, {"seed": 0, "fanout": 2}),
+                                            ("dbt", "allreduce", 8, {}), ("hm", "allreduce", 8, {"g": 4})])
+def test_flag_rings_per_sending_lane(name, coll, n, kw):
+    """R26: with the device's flag encoding (slot pos % K overwritten with pos + 1, the
+    receiver tests slot >= pos + 1), one ring per link is wrong under the direct
+    transport -- a pull-send posts without a credit wait, and a link fed by two lanes
+    (a fused forward beside a plain send) can post out of order: the receiver sees a
+    position early or loses one.  One ring per (link, sending lane) makes the device
+    test agree with the ideal "posted" everywhere, for both transports."""
+    g = ir.generate(name, coll, n, **kw)
+    for direct in (False, True):
+        p = lower.lower(g, "pair", direct=direct)
+        link_bad = 0
+        for K in (1, 2):
+            for n_mb in (1, 2, 3):
+                for sched, seed in (("rr", 0), ("random", 1), ("random", 2)):
+                    s = replay._Sim(p, n_mb, 1, K, rings="lane")
+                    s.run(sched, seed)
+                    assert s.hazards == [], (direct, K, n_mb, sched, s.hazards[:3])
+                    s = replay._Sim(p, n_mb, 1, K, rings="link")
+                    s.run(sched, seed)
+                    link_bad += bool(s.hazards)
+                    if not direct:
+                        assert s.hazards == []  # staged: the FIFO credit orders every post
+        if direct and name in ("ring", "synth"):
+            assert link_bad > 0  # the per-link encoding is observably broken here
