@@ -50,7 +50,7 @@ def parse():
     p.add_argument("--fifo-depth", type=int, default=0)
     p.add_argument("--nwarps", type=int, default=0)
     p.add_argument("--tma", type=int, default=-1, help="-1 = library default (on)")
-    p.add_argument("--direct", type=int, default=-1, help="direct push/pull transport (N=1 virtual ranks)")
+    p.add_argument("--direct", type=int, default=-1, help="direct push/pull transport (default 1; N>1 registers a symmetric window)")
     p.add_argument("--e2e-steps", type=int, default=3)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--sweep", default="", help="comma-separated MiB sizes for an extra busBW sweep")
@@ -218,11 +218,11 @@ def main():
     # default tuning: fill the SMs at N=1 (8 virtual ranks share one GPU)
     # default tuning (r01 sweeps, profiles/r01_*): 18 instances x 8 virtual ranks = 144 CTAs
     # (of 148 SMs), 4 MiB transfer chunks, FIFO depth 2 (FIFOs stay L2-resident)
-    # N=1: every virtual rank's buffers share one address space, so the direct transport
-    # (R23: push recv payloads, pull rrc operands; no FIFO staging) is the default there;
-    # multi-process (N>1) communicators use the staged FIFO transport.
+    # The direct transport (R23: push recv payloads, pull rrc operands; no FIFO staging) is
+    # the default: at N=1 every virtual rank's buffers share one address space; under
+    # torchrun (N>1) the send and receive buffers sit in a registered symmetric window.
     inst = args.instances or 18
-    direct = (0 if multi else 1) if args.direct < 0 else args.direct
+    direct = 1 if args.direct < 0 else args.direct
     opts = {"instances": inst, "chunkbytes": args.chunk_bytes or ((8 << 20) if direct else (4 << 20)),
             "fifodepth": args.fifo_depth or 2,
             "nwarps": args.nwarps or None, "tma": None if args.tma < 0 else args.tma,
@@ -248,6 +248,13 @@ def main():
              if tdt.is_floating_point else torch.randint(-2 ** 20, 2 ** 20, (count,), device=dev, dtype=tdt)
              for r in my_ranks}
     recvs = {r: torch.empty_like(sends[r]) for r in my_ranks}
+    if multi and direct:
+        # symmetric window: [send | pad | recv] at the same offsets on every rank
+        pad = 256 // elt
+        win = torch.empty(2 * count + pad, dtype=tdt, device=dev)
+        win[:count].copy_(sends[rank])
+        sends[rank], recvs[rank] = win[:count], win[count + pad:2 * count + pad]
+        comm.register(win)
     stream = torch.cuda.current_stream(dev)
     sid = stream.cuda_stream
 

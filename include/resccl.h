@@ -194,6 +194,18 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
 /* Control-only blocking simulation of a planned IR (invariant I4): *ok = 1 if the
  * plan completes for FIFO depth K and n_mb micro-batches. */
 rescclResult_t rescclCheckDeadlock(const char* irText, const char* opts, int K, int n_mb, int* ok);
+/* Wall-clock timeline of a planned IR under the alpha-beta model with link contention
+ * (Eq. 1; task-level execution, Eq. 5; reading R27), and the
+ * state-based merge of Eq. 7 evaluated on wall-clock activity active_l(t)
+ * (P:L1852-1885).  `params`: "count=<elements per rank buffer> elt=<2|4> alpha=<s>
+ * beta=<s/byte> gamma=<s>"; the micro-batch geometry follows the plan's chunkbytes
+ * and instances (`opts` / IR header), K = fifodepth.  Writes JSON: makespan_s,
+ * comm_time / avg_idle / max_idle over lanes (Table 3's metrics, predicted), the
+ * largest contention z, and per rank the connections' activity intervals and the
+ * merged lane counts (wall clock vs pipeline index).  InvalidUsage if the plan
+ * deadlocks. */
+rescclResult_t rescclSimulateTimeline(const char* irText, const char* opts, const char* params, char* json,
+                                      size_t* len);
 
 #ifdef __cplusplus
 }

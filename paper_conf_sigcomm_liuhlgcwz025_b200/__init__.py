@@ -46,7 +46,7 @@ EXPORTS = [
     "rescclAllReduce",
     "rescclAllGather", "rescclReduceScatter", "rescclGenerateIr", "rescclPlanIr",
     "rescclCodegenIr", "rescclCompileIr", "rescclCheckDeadlock", "rescclParseResCCLang", "rescclProfilePlanner",
-    "rescclCommRegister", "rescclCommRegisterConnect",
+    "rescclCommRegister", "rescclCommRegisterConnect", "rescclSimulateTimeline",
 ]
 
 _c = ctypes
@@ -72,6 +72,7 @@ _SIGS = {
     "rescclReduceScatter": (_i, [_vp, _vp, _sz, _i, _i, _vp, _vp]),
     "rescclGenerateIr": (_i, [_c.c_char_p, _i, _i, _c.c_char_p, _c.c_char_p, _c.POINTER(_sz)]),
     "rescclPlanIr": (_i, [_c.c_char_p, _c.c_char_p, _c.c_char_p, _c.POINTER(_sz)]),
+    "rescclSimulateTimeline": (_i, [_c.c_char_p, _c.c_char_p, _c.c_char_p, _c.c_char_p, _c.POINTER(_sz)]),
     "rescclCodegenIr": (_i, [_c.c_char_p, _c.c_char_p, _i, _i, _c.c_char_p, _c.POINTER(_sz)]),
     "rescclCompileIr": (_i, [_c.c_char_p, _c.c_char_p, _i, _i, _c.POINTER(_sz)]),
     "rescclCheckDeadlock": (_i, [_c.c_char_p, _c.c_char_p, _i, _i, _c.POINTER(_i)]),
@@ -255,6 +256,12 @@ def rescclProfilePlanner(program: str, opts: str = "", verify: bool = False) -> 
 
 def rescclPlanIr(ir_text: str, opts: str = "") -> dict:
     return json.loads(_sized(_lib.rescclPlanIr, _b(ir_text), _b(opts)))
+
+
+def rescclSimulateTimeline(ir_text: str, opts: str = "", count: int = 1 << 20, elt: int = 2,
+                           alpha: float = 2e-6, beta: float = 1 / 900e9, gamma: float = 2e-6) -> dict:
+    params = f"count={count} elt={elt} alpha={alpha!r} beta={beta!r} gamma={gamma!r}"
+    return json.loads(_sized(_lib.rescclSimulateTimeline, _b(ir_text), _b(opts), _b(params)))
 
 
 def rescclCodegenIr(ir_text: str, opts: str = "", rank_lo: int = 0, rank_hi: Optional[int] = None) -> str:

@@ -30,10 +30,11 @@ SOURCES = [
     "plan/plan.cc",
     "plan/codegen.cc",
     "plan/rescclang.cc",
+    "plan/timeline.cc",
     "comm/comm.cc",
 ]
 HEADERS = [
-    "plan/ir.h", "plan/plan.h", "plan/codegen.h", "device/resccl_device.cuh",
+    "plan/ir.h", "plan/plan.h", "plan/codegen.h", "plan/timeline.h", "device/resccl_device.cuh",
 ]
 
 

@@ -26,6 +26,7 @@
 
 #include "../../../include/resccl.h"
 #include "../plan/codegen.h"
+#include "../plan/timeline.h"
 #include "../plan/ir.h"
 #include "../plan/plan.h"
 
@@ -1376,6 +1377,39 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
   }
   auto cub = nvrtc_compile(codegen(p, L, co), dtype, op, co.gpu_scope);
   if (cubin_bytes) *cubin_bytes = cub.size();
+  API_END
+}
+
+rescclResult_t rescclSimulateTimeline(const char* irText, const char* opts, const char* params, char* json,
+                                      size_t* len) {
+  API_BEGIN
+  Options o;
+  Plan p = plan_from(irText, opts, &o, nullptr);
+  TimelineParams tp;
+  long long count = 0;
+  int elt = 2;
+  for (auto& kv : parse_kv(params)) {
+    double v;
+    try {
+      v = std::stod(kv.second);
+    } catch (...) {
+      fail(rescclInvalidArgument, "timeline parameter " + kv.first + " is not a number");
+    }
+    if (kv.first == "alpha") tp.alpha = v;
+    else if (kv.first == "beta") tp.beta = v;
+    else if (kv.first == "gamma") tp.gamma = v;
+    else if (kv.first == "count") count = (long long)v;
+    else if (kv.first == "elt") elt = (int)v;
+    else fail(rescclInvalidArgument, "unknown timeline parameter " + kv.first);
+  }
+  if (count <= 0 || (elt != 2 && elt != 4)) fail(rescclInvalidArgument, "timeline needs count > 0 and elt 2|4");
+  Geometry g = geometry(p.ir.coll, p.ir.nranks, count, elt, o.chunk_bytes, o.instances);
+  tp.n_mb = g.n_mb;
+  tp.c = (double)g.Mi * elt;
+  tp.K = o.fifo_depth;
+  tp.instances = o.instances;
+  TimelineResult r = simulate_timeline(p, tp);
+  write_out(timeline_json(p, tp, r), json, len);
   API_END
 }
 
