@@ -221,11 +221,18 @@ def main():
     # The direct transport (R23: push recv payloads, pull rrc operands; no FIFO staging) is
     # the default: at N=1 every virtual rank's buffers share one address space; under
     # torchrun (N>1) the send and receive buffers sit in a registered symmetric window.
-    inst = args.instances or 18
+    # N=1 (r01 tunes, profiles/r01_pool_tune.txt): two 256-thread CTAs per SM on all 148
+    # SMs (37 instances x 8 ranks = 296 CTAs), each with a 4-stage pool of 24 KiB TMA
+    # stages shared by its two lanes, and 32 MiB transfer chunks (one micro-batch per
+    # 32 MiB algorithm chunk).
     direct = 1 if args.direct < 0 else args.direct
-    opts = {"instances": inst, "chunkbytes": args.chunk_bytes or ((8 << 20) if direct else (4 << 20)),
+    two_per_sm = direct and not multi and not args.instances and not args.nwarps
+    inst = args.instances or (37 if two_per_sm else 18)
+    opts = {"instances": inst,
+            "chunkbytes": args.chunk_bytes or ((32 << 20) if two_per_sm else (8 << 20) if direct else (4 << 20)),
             "fifodepth": args.fifo_depth or 2,
-            "nwarps": args.nwarps or None, "tma": None if args.tma < 0 else args.tma,
+            "nwarps": args.nwarps or (8 if two_per_sm else None), "tma": None if args.tma < 0 else args.tma,
+            "tmastages": 2 if two_per_sm else None, "tmatile": 12288 if two_per_sm else None,
             "direct": direct}
     text = ir_text(R, args.algo, n, opts)
 
@@ -399,7 +406,9 @@ def main():
         cpu = {"value": round(bus_cpu, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc,
                "s_per_call": round(dt_cpu, 3)}
 
-    sms = sum(blocks) if not multi else blocks[rank]
+    # SMs the kernel occupies: its CTAs (one or two per SM, by block size) spread over the SMs
+    n_sm = torch.cuda.get_device_properties(dev).multi_processor_count
+    sms = min(n_sm, sum(blocks) if not multi else blocks[rank])
     line = {
         "metric": "allreduce busBW", "value": round(busbw, 2), "unit": "GB/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,

@@ -142,6 +142,7 @@ struct Options {
   int backoff = 1;
   int jitter = 0;
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
+  int pool_cap = 0;  // stages of the CTA pool one lane may hold (0 = all)
   int sys_rank = -1; // rescclCompileIr / rescclCodegenIr: one rank's multi-process (.sys) kernel
 };
 
@@ -187,6 +188,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "backoff") o.backoff = (int)to_long(v, k);
   else if (k == "jitter") o.jitter = (int)to_long(v, k);
   else if (k == "sysrank") o.sys_rank = (int)to_long(v, k);
+  else if (k == "poolcap") o.pool_cap = (int)to_long(v, k);
   else if (k == "sched") {
     if (v == "hpds") o.sched = 0;
     else if (v == "rr") o.sched = 1;
@@ -488,6 +490,7 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.backoff = a.opt.backoff;
   co.jitter = a.opt.jitter;
   co.exit_barrier = a.opt.direct && !gpu_scope;
+  co.pool_cap = a.opt.pool_cap;
   std::string src = codegen(a.plan, a.lay, co);
   if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
     if (FILE* f = fopen((std::string(dump) + "_" + a.ir.name + "_" + coll_name(a.ir.coll) + ".cu").c_str(), "w")) {

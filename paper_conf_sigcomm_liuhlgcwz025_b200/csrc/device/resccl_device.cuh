@@ -125,6 +125,14 @@ __device__ __forceinline__ void nanosleep_(u32 ns) {
 struct V4 {
   u32 x, y, z, w;
 };
+__device__ __forceinline__ V4 lds_v4(u32 a) {
+  V4 v;
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_v4(u32 a, const V4& v) {
+  asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
 __device__ __forceinline__ V4 ld_cg(const V4* p) {
   V4 v;
   asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
@@ -160,6 +168,33 @@ __device__ __forceinline__ void st_b16(void* p, u16 v) { asm volatile("st.global
 __device__ __forceinline__ u32 smem_u32(const void* p) {
   return (u32)__cvta_generic_to_shared(p);
 }
+// shared-memory state through 32-bit shared addresses (generic pointers would compile to
+// generic strong loads / GPU-scope atomics)
+__device__ __forceinline__ u32 lds_u32(u32 a) {
+  u32 v;
+  asm volatile("ld.volatile.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_u32(u32 a, u32 v) {
+  asm volatile("st.volatile.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ u32 lds_u8(u32 a) {
+  u32 v;
+  asm volatile("ld.volatile.shared.u8 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_u8(u32 a, u32 v) {
+  asm volatile("st.volatile.shared.u8 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ u32 atoms_and(u32 a, u32 v) {
+  u32 old;
+  asm volatile("atom.shared.and.b32 %0, [%1], %2;" : "=r"(old) : "r"(a), "r"(v) : "memory");
+  return old;
+}
+__device__ __forceinline__ void atoms_or(u32 a, u32 v) {
+  asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void fence_cta() { asm volatile("fence.acq_rel.cta;" ::: "memory"); }
 __device__ __forceinline__ void mbar_init(u32 bar, u32 count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
 }
@@ -186,7 +221,7 @@ __device__ __forceinline__ void mbar_arrive(u32 bar) {
 __device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 // wait until at most n bulk groups are pending (n must be an immediate)
 __device__ __forceinline__ void tma_wait_n(u32 n) {
-  switch (n) {
+  switch (n < 15 ? n : 15) {
     case 1: asm volatile("cp.async.bulk.wait_group 1;" ::: "memory"); break;
     case 2: asm volatile("cp.async.bulk.wait_group 2;" ::: "memory"); break;
     case 3: asm volatile("cp.async.bulk.wait_group 3;" ::: "memory"); break;
@@ -194,11 +229,19 @@ __device__ __forceinline__ void tma_wait_n(u32 n) {
     case 5: asm volatile("cp.async.bulk.wait_group 5;" ::: "memory"); break;
     case 6: asm volatile("cp.async.bulk.wait_group 6;" ::: "memory"); break;
     case 7: asm volatile("cp.async.bulk.wait_group 7;" ::: "memory"); break;
+    case 8: asm volatile("cp.async.bulk.wait_group 8;" ::: "memory"); break;
+    case 9: asm volatile("cp.async.bulk.wait_group 9;" ::: "memory"); break;
+    case 10: asm volatile("cp.async.bulk.wait_group 10;" ::: "memory"); break;
+    case 11: asm volatile("cp.async.bulk.wait_group 11;" ::: "memory"); break;
+    case 12: asm volatile("cp.async.bulk.wait_group 12;" ::: "memory"); break;
+    case 13: asm volatile("cp.async.bulk.wait_group 13;" ::: "memory"); break;
+    case 14: asm volatile("cp.async.bulk.wait_group 14;" ::: "memory"); break;
+    case 15: asm volatile("cp.async.bulk.wait_group 15;" ::: "memory"); break;
     default: asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); break;
   }
 }
 __device__ __forceinline__ void tma_wait_read_n(u32 n) {
-  switch (n) {
+  switch (n < 15 ? n : 15) {
     case 1: asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); break;
     case 2: asm volatile("cp.async.bulk.wait_group.read 2;" ::: "memory"); break;
     case 3: asm volatile("cp.async.bulk.wait_group.read 3;" ::: "memory"); break;
@@ -206,6 +249,14 @@ __device__ __forceinline__ void tma_wait_read_n(u32 n) {
     case 5: asm volatile("cp.async.bulk.wait_group.read 5;" ::: "memory"); break;
     case 6: asm volatile("cp.async.bulk.wait_group.read 6;" ::: "memory"); break;
     case 7: asm volatile("cp.async.bulk.wait_group.read 7;" ::: "memory"); break;
+    case 8: asm volatile("cp.async.bulk.wait_group.read 8;" ::: "memory"); break;
+    case 9: asm volatile("cp.async.bulk.wait_group.read 9;" ::: "memory"); break;
+    case 10: asm volatile("cp.async.bulk.wait_group.read 10;" ::: "memory"); break;
+    case 11: asm volatile("cp.async.bulk.wait_group.read 11;" ::: "memory"); break;
+    case 12: asm volatile("cp.async.bulk.wait_group.read 12;" ::: "memory"); break;
+    case 13: asm volatile("cp.async.bulk.wait_group.read 13;" ::: "memory"); break;
+    case 14: asm volatile("cp.async.bulk.wait_group.read 14;" ::: "memory"); break;
+    case 15: asm volatile("cp.async.bulk.wait_group.read 15;" ::: "memory"); break;
     default: asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); break;
   }
 }
@@ -427,13 +478,17 @@ struct Lane {
   char* self;       // this rank's plan region
   int rank, inst, bar, nthreads, tid;
   volatile int* abort_flag;  // shared memory, per lane
-  char* stage;               // this lane's TMA staging: RESCCL_TMA_STAGES x (A tile, B tile)
-  u32 full;                  // shared address of the "tile loaded" mbarriers (one per stage)
-  u32 comp;                  // shared address of the "tile combined" mbarriers (one per stage)
-  u32 tseq;                  // tiles streamed so far by this lane: stage = tseq % S, parity = tseq / S
-  u32 comp_use[RESCCL_TMA_STAGES];  // leader: completed phases of each comp barrier
-  volatile u32* issued;      // shared: tiles the leader has issued (combine warps must not test a
+  // shared-memory addresses (32-bit):
+  u32 stage;                 // the CTA's stage pool: RESCCL_POOL x (A tile, B tile), shared by both lanes
+  u32 full;                  // "tile loaded" mbarriers (one per pool stage)
+  u32 comp;                  // "tile combined" mbarriers (one per pool stage)
+  u32 pool;                  // u32 mask: bit s set = pool stage s free
+  u32 fuse, cuse;            // u32[POOL]: completed phases of full[s] / comp[s] (owner-updated)
+  u32 qst, qpar;             // u8[QN], this lane: stage of tile k (k % QN) and its full parity,
+                             // for the combine warps
+  u32 issued;                // u32: tiles the leader has issued (combine warps must not test a
                              // stage's parity before its tile is issued: no ABA on phases)
+  u32 tseq;                  // tiles streamed so far by this lane
   u64 wait_ns;               // RESCCL_TRACE: leader time spent waiting (idle ratio, Table 3)
 
   __device__ __forceinline__ void sync() const {
@@ -619,6 +674,38 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
   return true;
 }
 
+// The two lanes of a CTA draw TMA stages from one pool (RESCCL_POOL = 2 x
+// RESCCL_TMA_STAGES stages): in most schedules only one lane moves data at a time (ring
+// AllReduce: the receive lane during ReduceScatter, the send lane during AllGather),
+// so a shared pool doubles the bytes in flight of the active lane.  A leader claims a
+// stage only for a tile it issues at once, and every held stage frees itself without
+// any remote condition (load lands, combine warps finish, the store reads it out, the
+// micro-batch posts -- posting waits only for its own stores).  A leader waiting on a
+// remote condition has posted everything it loaded, so it holds no stage; a lane
+// waiting for a stage waits only for the other lane's in-flight tiles: no new wait edge.
+#define RESCCL_POOL (2 * RESCCL_TMA_STAGES)
+#ifndef RESCCL_POOL_CAP
+#define RESCCL_POOL_CAP RESCCL_POOL  // stages one lane may hold
+#endif
+#define RESCCL_QN 32
+__device__ __forceinline__ int pool_claim(u32 pool) {
+  u32 m = lds_u32(pool);
+  while (m) {
+    const int s = __ffs(m) - 1;
+    const u32 old = atoms_and(pool, ~(1u << s));
+    if (old & (1u << s)) {
+      fence_cta();
+      return s;
+    }
+    m = old & ~(1u << s);
+  }
+  return -1;
+}
+__device__ __forceinline__ void pool_release(u32 pool, int s) {
+  fence_cta();
+  atoms_or(pool, 1u << s);
+}
+
 // Number of TMA tiles of micro-batch j (16-byte-aligned body only).  A stage holds one
 // reduce tile (A and B halves of RESCCL_TMA_TILE bytes) or one copy tile of twice that.
 template <int F>
@@ -641,16 +728,21 @@ __device__ __forceinline__ u32 mb_tiles(const KArgs& a, i64 len, int j, int inst
 template <class T, int OP, int F>
 __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
   const KArgs& a = *L.a;
-  const int NS = RESCCL_TMA_STAGES;
+  const u32 P = RESCCL_POOL;
   const i64 TB = tile_bytes<F>();
   const int nmb = a.n_mb;
   const u32 k0 = L.tseq;
-  const u32 sbase = smem_u32(L.stage);
+  const u32 sbase = L.stage;
   const u64 mb_base = a.mb_base;
   int rj = 0;                 // micro-batches whose readiness is confirmed
   int lj = 0;                 // load cursor (micro-batch, tile)
   u32 lt = 0;
-  u32 issued = 0, stored = 0; // tiles
+  u32 issued = 0, stored = 0, released = 0;  // tiles
+  // per in-flight tile (slot = tile % P), kept in registers: its stage (4 bits) and the
+  // parities of its full / comp barrier phases (1 bit each)
+  u64 hs = 0;
+  u32 hf = 0, hc = 0;
+#define RESCCL_HS(slot) ((u32)(hs >> (4 * (slot))) & 15u)
   int sj = 0;                 // store cursor
   u32 st = 0;
   int pj = 0;                 // next micro-batch to post
@@ -707,10 +799,30 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
         if (lj < nmb) T_l = mb_tiles<F>(a, p.len, lj, L.inst, T::kSize, lo_l, nb_l);
         continue;
       }
-      if (issued - stored >= (u32)NS) break;
-      if (issued >= (u32)NS) tma_wait_read_n(stored - 1 - (issued - NS));  // stage's last store read smem
+      int sc = (issued - released < (u32)RESCCL_POOL_CAP) ? pool_claim(L.pool) : -1;
+      if (sc < 0 && stored > released) {  // recycle our oldest stored stage (its store read it out)
+        const u32 keep = stored - released - 1 < 15 ? stored - released - 1 : 15;
+        tma_wait_read_n(keep);
+        const u32 upto = stored - keep;
+        for (; released < upto; ++released) pool_release(L.pool, RESCCL_HS(released % P));
+        if (issued - released < (u32)RESCCL_POOL_CAP) sc = pool_claim(L.pool);
+      }
+      if (sc < 0) break;  // the other lane holds the pool: its tiles drain by themselves
+      const u32 s = (u32)sc;
       const u32 k = k0 + issued;
-      const u32 s = k % NS;
+      const u32 slot = issued % P;
+      const u32 fu = lds_u32(L.fuse + 4 * s);
+      const u32 fpar = fu & 1;
+      hs = (hs & ~(15ull << (4 * slot))) | ((u64)s << (4 * slot));
+      hf = (hf & ~(1u << slot)) | (fpar << slot);
+      sts_u32(L.fuse + 4 * s, fu + 1);
+      if (F & kReduce) {
+        const u32 cu = lds_u32(L.cuse + 4 * s);
+        hc = (hc & ~(1u << slot)) | ((cu & 1) << slot);
+        sts_u32(L.cuse + 4 * s, cu + 1);
+        sts_u8(L.qst + k % RESCCL_QN, s);
+        sts_u8(L.qpar + k % RESCCL_QN, fpar);
+      }
       const i64 off = (i64)lt * TB;
       const u32 nb = (u32)((nb_l - off) < TB ? (nb_l - off) : TB);
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
@@ -734,15 +846,18 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       }
       ++issued;
       ++lt;
-      if (F & kReduce) *L.issued = k0 + issued;
+      if (F & kReduce) {
+        fence_cta();  // qst / qpar before the issued count
+        sts_u32(L.issued, k0 + issued);
+      }
       prog = true;
     }
     // (3) stores
     while (stored < issued) {
-      const u32 k = k0 + stored;
-      const u32 s = k % NS;
-      const bool ok = (F & kReduce) ? mbar_test(L.comp + 8 * s, L.comp_use[s] & 1)
-                                    : mbar_test(L.full + 8 * s, (k / NS) & 1);
+      const u32 slot = stored % P;
+      const u32 s = RESCCL_HS(slot);
+      const bool ok = (F & kReduce) ? mbar_test(L.comp + 8 * s, (hc >> slot) & 1)
+                                    : mbar_test(L.full + 8 * s, (hf >> slot) & 1);
       if (!ok) break;
       while (st >= T_s) {
         ++sj;
@@ -762,7 +877,6 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
         }
       }
       tma_commit();
-      if (F & kReduce) L.comp_use[s]++;
       ++stored;
       ++st;
       prog = true;
@@ -770,6 +884,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
     // (4) post
     if (pj < rj && stored >= gp_end) {
       tma_wait_n(stored - gp_end);
+      for (; released < gp_end; ++released) pool_release(L.pool, RESCCL_HS(released % P));  // written out
       // unaligned tail (< 16 bytes) of this micro-batch: scalar, by the leader
       i64 lo_h, hi_h;
       slice_of(a, p.len, pj, L.inst, lo_h, hi_h);
@@ -818,6 +933,11 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       }
     }
   }
+  if (stored > released) {  // (all posted: every store has completed)
+    tma_wait_read_n(0);
+    for (; released < stored; ++released) pool_release(L.pool, RESCCL_HS(released % P));
+  }
+#undef RESCCL_HS
 #if RESCCL_TRACE
   if (t_idle) L.wait_ns += globaltimer() - t_idle;
 #endif
@@ -830,28 +950,29 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
 template <class T, int OP, int F>
 __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const PrimPtrs& p, int ctid, int nct) {
   const KArgs& a = *L.a;
-  const int NS = RESCCL_TMA_STAGES;
   const i64 TB = RESCCL_TMA_TILE;  // reduce tiles only
   u32 k = L.tseq;
   for (int j = 0; j < a.n_mb; ++j) {
     i64 lo, nbj;
     const u32 ntl = mb_tiles<F>(a, p.len, j, L.inst, T::kSize, lo, nbj);
     for (u32 t = 0; t < ntl; ++t, ++k) {
-      const u32 s = k % NS;
       const i64 off = (i64)t * TB;
       const int nb = (int)((nbj - off) < TB ? (nbj - off) : TB);
       u32 spins = 0;
-      while ((int)(*L.issued - k) <= 0) {  // tile k not issued yet
+      while ((int)(lds_u32(L.issued) - k) <= 0) {  // tile k not issued yet
         if (++spins > 16) nanosleep_(20);
         if ((spins & 1023) == 0 && *L.abort_flag) return false;
       }
-      while (!mbar_test(L.full + 8 * s, (k / NS) & 1)) {
+      fence_cta();
+      const u32 s = lds_u8(L.qst + k % RESCCL_QN);
+      const u32 par = lds_u8(L.qpar + k % RESCCL_QN);
+      while (!mbar_test(L.full + 8 * s, par)) {
         if (++spins > 16) nanosleep_(20);
         if ((spins & 1023) == 0 && *L.abort_flag) return false;
       }
-      V4* av = (V4*)(L.stage + (i64)s * 2 * TB);
-      const V4* bv = (const V4*)(L.stage + (i64)s * 2 * TB + TB);
-      for (int i = ctid; i < nb / 16; i += nct) av[i] = combine_v<T, OP>(av[i], bv[i]);
+      const u32 sa = L.stage + s * 2 * (u32)TB;
+      for (int i = ctid; i < nb / 16; i += nct)
+        sts_v4(sa + 16 * i, combine_v<T, OP>(lds_v4(sa + 16 * i), lds_v4(sa + (u32)TB + 16 * i)));
       fence_proxy_async_smem();
       __syncwarp();
       if ((threadIdx.x & 31) == 0) mbar_arrive(L.comp + 8 * s);

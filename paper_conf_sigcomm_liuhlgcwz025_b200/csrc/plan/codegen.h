@@ -57,13 +57,16 @@ struct CodegenOpts {
   int backoff = 1;               // nanosleep back-off while polling flags
   int jitter = 0;                // debug fault injector: random delays around every sync
   int prefetch = 0;              // micro-batches of local operand prefetched into L2 ahead (off: r01)
+  int pool_cap = 0;              // stages of the CTA pool one lane may hold (0 = all)
   int exit_barrier = 0;          // direct transport across processes: a rank's kernel ends only
                                  // after every peer's blocks finished touching its buffers
 };
 
 // dynamic shared memory the generated kernel needs (both lanes' TMA staging)
-// (2 lanes x stages x (A tile + B tile))
-inline int codegen_smem_bytes(const CodegenOpts& o) { return o.tma ? 4 * o.tma_stages * o.tma_tile : 0; }
+// (a pool of 2 x stages stages of (A tile + B tile), shared by the CTA's two lanes)
+inline int codegen_smem_bytes(const CodegenOpts& o) {
+  return o.tma ? 4 * o.tma_stages * o.tma_tile : 0;
+}
 
 // Device code (without the L0 library text, which the runtime prepends).
 std::string codegen(const Plan& p, const Layout& L, const CodegenOpts& o);
