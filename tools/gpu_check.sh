@@ -1,0 +1,9 @@
+# Round-end style check on one B200: smoke, the -m gpu suite, the default bench line.
+mkdir -p gpurun_out
+export RESCCL_TIMEOUT_MS=20000
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1
+echo "pytest=$?" >> gpurun_out/pytest_gpu.log
+python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
+tail -3 gpurun_out/pytest_gpu.log
+cat gpurun_out/bench_default.json
