@@ -143,6 +143,8 @@ struct Options {
   int jitter = 0;
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
   int pool_cap = 0;  // stages of the CTA pool one lane may hold (0 = all)
+  int ring = 0;      // lane-private TMA stage rings (1) vs one pool shared by both lanes (0)
+  int store_lag = 1; // bulk stores a lane lets drain before it blocks to reuse a stage
   int sys_rank = -1; // rescclCompileIr / rescclCodegenIr: one rank's multi-process (.sys) kernel
 };
 
@@ -189,6 +191,8 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "jitter") o.jitter = (int)to_long(v, k);
   else if (k == "sysrank") o.sys_rank = (int)to_long(v, k);
   else if (k == "poolcap") o.pool_cap = (int)to_long(v, k);
+  else if (k == "storelag") o.store_lag = (int)to_long(v, k);
+  else if (k == "ring") o.ring = (int)to_long(v, k);
   else if (k == "sched") {
     if (v == "hpds") o.sched = 0;
     else if (v == "rr") o.sched = 1;
@@ -209,7 +213,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -220,6 +224,8 @@ Options make_options(const Ir& ir, const char* extra) {
   if (o.tma_tile < 1024 || o.tma_tile % 128 || o.tma_stages < 1 || o.tma_stages > 8 ||
       4 * o.tma_tile * o.tma_stages > 200 * 1024)
     fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 4*tile*stages <= 200 KiB");
+  if (o.store_lag < 1 || o.store_lag > o.tma_stages)
+    fail(rescclInvalidArgument, "storelag must be 1..tmastages");
   return o;
 }
 
@@ -469,28 +475,37 @@ std::string info_json(const AlgoShared& a) {
 // use_tma: the call's instance slices reach `tmamin` bytes; otherwise a variant without
 // the TMA engine (no dynamic shared memory, no mbarrier setup) is launched -- small
 // messages are latency-bound and the staging only costs launch overhead there.
+// codegen options carried by an Options set (every kernel-build path uses this)
+CodegenOpts codegen_opts(const Options& o) {
+  CodegenOpts co;
+  co.nwarps = o.nwarps;
+  co.tma = o.tma;
+  co.tma_tile = o.tma_tile;
+  co.tma_stages = o.tma_stages;
+  co.trace = o.trace;
+  co.l2hint = o.l2hint;
+  co.prefetch = o.prefetch;
+  co.tma_min = o.tma_min;
+  co.backoff = o.backoff;
+  co.jitter = o.jitter;
+  co.pool_cap = o.pool_cap;
+  co.store_lag = o.store_lag;
+  co.ring = o.ring;
+  return co;
+}
+
 Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, int hi, bool gpu_scope,
                  bool use_tma) {
   std::string key = std::to_string((int)dt) + "/" + std::to_string((int)op) + "/" + std::to_string(lo) + "-" +
                     std::to_string(hi) + "/" + (gpu_scope ? "g" : "s") + (use_tma ? "/t" : "/n");
   auto it = a.kernels.find(key);
   if (it != a.kernels.end()) return it->second;
-  CodegenOpts co;
+  CodegenOpts co = codegen_opts(a.opt);
   co.rank_lo = lo;
   co.rank_hi = hi;
   co.gpu_scope = gpu_scope;
-  co.nwarps = a.opt.nwarps;
   co.tma = use_tma ? a.opt.tma : 0;
-  co.tma_tile = a.opt.tma_tile;
-  co.tma_stages = a.opt.tma_stages;
-  co.trace = a.opt.trace;
-  co.l2hint = a.opt.l2hint;
-  co.prefetch = a.opt.prefetch;
-  co.tma_min = a.opt.tma_min;
-  co.backoff = a.opt.backoff;
-  co.jitter = a.opt.jitter;
   co.exit_barrier = a.opt.direct && !gpu_scope;
-  co.pool_cap = a.opt.pool_cap;
   std::string src = codegen(a.plan, a.lay, co);
   if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
     if (FILE* f = fopen((std::string(dump) + "_" + a.ir.name + "_" + coll_name(a.ir.coll) + ".cu").c_str(), "w")) {
@@ -1286,10 +1301,9 @@ rescclResult_t rescclProfilePlanner(const char* program, const char* opts, int v
   auto t3 = clk::now();
   Plan p = lower(ir, o.model, false, &pr, o.direct != 0);  // Lowering (translation + TB allocation)
   Layout L = make_layout(p, o.fifo_depth, o.instances, o.chunk_bytes);
-  CodegenOpts co;
+  CodegenOpts co = codegen_opts(o);
   co.rank_lo = 0;
   co.rank_hi = 1;
-  co.nwarps = o.nwarps;
   std::string src = codegen(p, L, co);              // kernel source of rank 0
   auto t4 = clk::now();
   bool ok = true;
@@ -1334,19 +1348,9 @@ rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo
   Plan p = plan_from(irText, opts, &o, nullptr);
   if (rank_lo < 0 || rank_hi > p.ir.nranks || rank_lo >= rank_hi) fail(rescclInvalidArgument, "bad rank range");
   Layout L = make_layout(p, o.fifo_depth, o.instances, o.chunk_bytes);
-  CodegenOpts co;
+  CodegenOpts co = codegen_opts(o);
   co.rank_lo = rank_lo;
   co.rank_hi = rank_hi;
-  co.nwarps = o.nwarps;
-  co.tma = o.tma;
-  co.tma_tile = o.tma_tile;
-  co.tma_stages = o.tma_stages;
-  co.trace = o.trace;
-  co.l2hint = o.l2hint;
-  co.prefetch = o.prefetch;
-  co.tma_min = o.tma_min;
-  co.backoff = o.backoff;
-  co.jitter = o.jitter;
   write_out(codegen(p, L, co), src, len);
   API_END
 }
@@ -1357,19 +1361,9 @@ rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataT
   Options o;
   Plan p = plan_from(irText, opts, &o, nullptr);
   Layout L = make_layout(p, o.fifo_depth, o.instances, o.chunk_bytes);
-  CodegenOpts co;
+  CodegenOpts co = codegen_opts(o);
   co.rank_lo = 0;
   co.rank_hi = p.ir.nranks;
-  co.nwarps = o.nwarps;
-  co.tma = o.tma;
-  co.tma_tile = o.tma_tile;
-  co.tma_stages = o.tma_stages;
-  co.trace = o.trace;
-  co.l2hint = o.l2hint;
-  co.prefetch = o.prefetch;
-  co.tma_min = o.tma_min;
-  co.backoff = o.backoff;
-  co.jitter = o.jitter;
   co.gpu_scope = true;
   if (o.sys_rank >= 0) {  // one rank of a multi-process communicator
     if (o.sys_rank >= p.ir.nranks) fail(rescclInvalidArgument, "sysrank out of range");

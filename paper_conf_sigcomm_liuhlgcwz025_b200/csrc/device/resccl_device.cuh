@@ -107,6 +107,20 @@ __device__ __forceinline__ u64 ld_acquire(const u64* p) {
 #endif
   return v;
 }
+// Polling: relaxed loads (an ld.acquire at .gpu/.sys scope compiles to a strong load plus
+// an L1 invalidate, CCTL.IVALL, on every spin), then one acquire load once the value is
+// reached: coherence makes it return a value >= the one observed, and it synchronises
+// with the producer's release (fence + store) of that value.
+__device__ __forceinline__ u64 ld_relaxed(const u64* p) {
+  u64 v;
+  asm volatile("ld.relaxed" RESCCL_SC ".global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ bool ready_ge(const u64* p, u64 target) {
+  if (ld_relaxed(p) < target) return false;
+  (void)ld_acquire(p);
+  return true;
+}
 __device__ __forceinline__ u64 globaltimer() {
   u64 t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -212,6 +226,16 @@ __device__ __forceinline__ bool mbar_test(u32 bar, u32 parity) {
   asm volatile(
       "{\n.reg .pred p;\n"
       "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      "selp.u32 %0, 1, 0, p;\n}\n" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
+  return ok != 0;
+}
+// one suspending wait: the warp sleeps in hardware until the phase completes or a
+// system-dependent time limit passes (no issue slots or smem bandwidth spent polling)
+__device__ __forceinline__ bool mbar_try(u32 bar, u32 parity) {
+  u32 ok;
+  asm volatile(
+      "{\n.reg .pred p;\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
       "selp.u32 %0, 1, 0, p;\n}\n" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
   return ok != 0;
 }
@@ -483,12 +507,12 @@ struct Lane {
   u32 full;                  // "tile loaded" mbarriers (one per pool stage)
   u32 comp;                  // "tile combined" mbarriers (one per pool stage)
   u32 pool;                  // u32 mask: bit s set = pool stage s free
-  u32 fuse, cuse;            // u32[POOL]: completed phases of full[s] / comp[s] (owner-updated)
-  u32 qst, qpar;             // u8[QN], this lane: stage of tile k (k % QN) and its full parity,
-                             // for the combine warps
-  u32 issued;                // u32: tiles the leader has issued (combine warps must not test a
-                             // stage's parity before its tile is issued: no ABA on phases)
+  u32 qprog;                 // u32: tiles this lane's leader announced to its combine warps
+  u32 qdesc;                 // u64: the current epoch (first tile | stage mask << 32 | parities << 48)
+  u32 want;                  // u32[2]: lane waits for pool stages (send lane, recv lane)
   u32 tseq;                  // tiles streamed so far by this lane
+  u32 ring0;                 // RESCCL_RING: first stage of this lane's private ring
+  u32 cpar;                  // RESCCL_RING (leader): comp-barrier phase parity per ring slot
   u64 wait_ns;               // RESCCL_TRACE: leader time spent waiting (idle ratio, Table 3)
 
   __device__ __forceinline__ void sync() const {
@@ -496,10 +520,10 @@ struct Lane {
   }
   // leader only: spin until *p >= target; false on timeout (error word set)
   __device__ bool wait_ge(const u64* p, u64 target) {
-    if (ld_acquire(p) >= target) return true;
+    if (ready_ge(p, target)) return true;
     u64 t0 = globaltimer();
     u32 spins = 0;
-    while (ld_acquire(p) < target) {
+    while (!ready_ge(p, target)) {
       if (++spins > 64) nanosleep_(32);
       if ((spins & 1023) == 0 && globaltimer() - t0 > a->timeout_ns) {
         atomicCAS(a->err, 0, kErrTimeout);
@@ -616,16 +640,16 @@ __device__ __forceinline__ bool mb_ready(const Lane& L, const PrimDesc& d, const
   const u64 mb_base = a.mb_base;
   if (!Kind<F>::push_recv)  // (a push receiver checked its dependencies when it posted "writable")
     for (int k = 0; k < d.ndeps; ++k)
-      if (ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) < dep_target(a, d, k, j)) return false;
+      if (!ready_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, j))) return false;
   if (F & kRecv) {
     const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
-    if (ld_acquire(p.in_flag + (in_seq % RESCCL_K)) < in_seq + 1) return false;
+    if (!ready_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1)) return false;
   }
   if (F & kSend) {
     const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
     if (F & kDirect) {
-      if (!(F & kSendPull) && ld_acquire(p.out_cred) < out_seq + 1) return false;  // push: writable
-    } else if (out_seq + 1 > (u64)RESCCL_K && ld_acquire(p.out_cred) < out_seq + 1 - RESCCL_K) {
+      if (!(F & kSendPull) && !ready_ge(p.out_cred, out_seq + 1)) return false;  // push: writable
+    } else if (out_seq + 1 > (u64)RESCCL_K && !ready_ge(p.out_cred, out_seq + 1 - RESCCL_K)) {
       return false;
     }
   }
@@ -674,42 +698,69 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
   return true;
 }
 
-// The two lanes of a CTA draw TMA stages from one pool (RESCCL_POOL = 2 x
-// RESCCL_TMA_STAGES stages): in most schedules only one lane moves data at a time (ring
-// AllReduce: the receive lane during ReduceScatter, the send lane during AllGather),
-// so a shared pool doubles the bytes in flight of the active lane.  A leader claims a
-// stage only for a tile it issues at once, and every held stage frees itself without
-// any remote condition (load lands, combine warps finish, the store reads it out, the
-// micro-batch posts -- posting waits only for its own stores).  A leader waiting on a
-// remote condition has posted everything it loaded, so it holds no stage; a lane
-// waiting for a stage waits only for the other lane's in-flight tiles: no new wait edge.
+// Stage management.  A CTA owns RESCCL_POOL = 2 x RESCCL_TMA_STAGES TMA stages (an A
+// and a B tile each).  In most schedules only one lane moves data at a time (ring
+// AllReduce: the receive lane during ReduceScatter, the send lane during AllGather), so
+// by default the lanes share the stages as a pool, claimed in *epochs*: a leader that has
+// confirmed-ready work and no stages takes every free stage (at most half while the other
+// lane waits for stages) with one shared-memory atomic, streams its tiles round-robin
+// through them, and returns them once everything it loaded is written out and no ready
+// work is left (or early, when the other lane waits and it holds more than half).
+// Per tile the leader touches shared memory only through the TMA, its mbarriers and one
+// progress word: its generic shared-memory operations queue behind the TMA's bulk smem
+// traffic (~300 cycles each under load), so per-tile claims capped the tile rate.
+// Deadlock freedom: a leader holds stages only while it has unposted tiles or confirmed-
+// ready loads, both of which complete without any remote condition, so a leader waiting
+// on a remote condition holds no stage and a lane waiting for stages waits only for the
+// other lane's local work: no new wait edge.
+// RESCCL_RING=1: each lane streams through a private ring of RESCCL_TMA_STAGES stages
+// instead (tile k -> stage ring0 + k % S, full parity (k / S) & 1).
 #define RESCCL_POOL (2 * RESCCL_TMA_STAGES)
 #ifndef RESCCL_POOL_CAP
 #define RESCCL_POOL_CAP RESCCL_POOL  // stages one lane may hold
 #endif
-#define RESCCL_QN 32
-__device__ __forceinline__ int pool_claim(u32 pool) {
-  u32 m = lds_u32(pool);
-  while (m) {
-    const int s = __ffs(m) - 1;
-    const u32 old = atoms_and(pool, ~(1u << s));
-    if (old & (1u << s)) {
-      fence_cta();
-      return s;
-    }
-    m = old & ~(1u << s);
-  }
-  return -1;
+#ifndef RESCCL_RING
+#define RESCCL_RING 0
+#endif
+// stores a lane lets drain before it blocks on the oldest to reuse its stage
+#ifndef RESCCL_STORE_LAG
+#define RESCCL_STORE_LAG 1
+#endif
+// parity of a quiescent mbarrier's current (incomplete) phase: the preceding phase, of
+// the other parity, tests complete
+__device__ __forceinline__ u32 mbar_phase(u32 bar) { return mbar_test(bar, 0) ? 1u : 0u; }
+__device__ __forceinline__ u64 lds_u64(u32 a) {
+  u64 v;
+  asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+  return v;
 }
-__device__ __forceinline__ void pool_release(u32 pool, int s) {
-  fence_cta();
-  atoms_or(pool, 1u << s);
+__device__ __forceinline__ void sts_u64(u32 a, u64 v) {
+  asm volatile("st.volatile.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+// i-th (0-based) set bit of m
+__device__ __forceinline__ u32 nth_bit(u32 m, u32 i) {
+  for (; i; --i) m &= m - 1;
+  return (u32)(__ffs(m) - 1);
 }
 
+__device__ __forceinline__ void slice_of_m(i64 M, i64 Mi, i64 len, int j, int inst, i64& lo, i64& hi) {
+  lo = (i64)j * M + (i64)inst * Mi;
+  hi = lo + Mi;
+  if (hi > (i64)(j + 1) * M) hi = (i64)(j + 1) * M;
+  if (hi > len) hi = len;
+  if (lo > hi) lo = hi;
+}
 // Number of TMA tiles of micro-batch j (16-byte-aligned body only).  A stage holds one
 // reduce tile (A and B halves of RESCCL_TMA_TILE bytes) or one copy tile of twice that.
 template <int F>
 __device__ __forceinline__ i64 tile_bytes() { return (F & kReduce) ? RESCCL_TMA_TILE : 2 * RESCCL_TMA_TILE; }
+template <int F>
+__device__ __forceinline__ u32 mb_tiles_m(i64 M, i64 Mi, i64 len, int j, int inst, int esz, i64& lo, i64& nb) {
+  i64 hi;
+  slice_of_m(M, Mi, len, j, inst, lo, hi);
+  nb = ((hi - lo) * esz) & ~(i64)15;
+  return (u32)((nb + tile_bytes<F>() - 1) / tile_bytes<F>());
+}
 template <int F>
 __device__ __forceinline__ u32 mb_tiles(const KArgs& a, i64 len, int j, int inst, int esz, i64& lo, i64& nb) {
   i64 hi;
@@ -719,7 +770,7 @@ __device__ __forceinline__ u32 mb_tiles(const KArgs& a, i64 len, int j, int inst
 }
 
 // TMA pipeline, leader thread: a non-blocking event loop that (1) confirms the
-// readiness of the next micro-batch, (2) streams its tiles into the stage ring with
+// readiness of the next micro-batch, (2) streams its tiles into its stages with
 // cp.async.bulk, (3) stores tiles whose data is loaded (copy) or combined (reduce) to
 // the local buffer and/or the peer FIFO, (4) posts a micro-batch once all its stores
 // completed.  It never blocks on a remote condition while it holds unposted work, so
@@ -728,7 +779,21 @@ __device__ __forceinline__ u32 mb_tiles(const KArgs& a, i64 len, int j, int inst
 template <class T, int OP, int F>
 __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
   const KArgs& a = *L.a;
-  const u32 P = RESCCL_POOL;
+  // Everything the loop reads per tile lives in registers: the lane, the arguments and
+  // the pointers are memory-resident (their addresses are taken), and every asm
+  // statement below clobbers memory, so field accesses would reload them each time.
+  const u32 Lfull = L.full, Lcomp = L.comp, Lpool = L.pool, Lqprog = L.qprog, Lqdesc = L.qdesc, Lwant = L.want;
+  const int Linst = L.inst, Lbar = L.bar;
+  const u32 Lring0 = L.ring0;
+  u32 Lcpar = L.cpar;
+  const i64 aM = a.M, aMi = a.Mi, plen = p.len;
+  const char* const pA = p.A;
+  const char* const pR = p.R;
+  char* const pQ = p.Q;
+  char* const pD1 = p.D1;
+  char* const pin = p.in_data;
+  char* const pout = p.out_data;
+  const u32 P = RESCCL_POOL;  // slots of the per-tile register records (>= stages held)
   const i64 TB = tile_bytes<F>();
   const int nmb = a.n_mb;
   const u32 k0 = L.tseq;
@@ -737,17 +802,29 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   int rj = 0;                 // micro-batches whose readiness is confirmed
   int lj = 0;                 // load cursor (micro-batch, tile)
   u32 lt = 0;
-  u32 issued = 0, stored = 0, released = 0;  // tiles
+  u32 issued = 0, stored = 0, released = 0;  // tiles (released: stage read out by its store)
   // per in-flight tile (slot = tile % P), kept in registers: its stage (4 bits) and the
   // parities of its full / comp barrier phases (1 bit each)
   u64 hs = 0;
   u32 hf = 0, hc = 0;
 #define RESCCL_HS(slot) ((u32)(hs >> (4 * (slot))) & 15u)
+#if RESCCL_RING
+  const u32 eR = RESCCL_TMA_STAGES;
+#else
+  u32 emask = 0, eR = 0;      // the epoch's stages (bit mask, count)
+  u64 ering = 0;              // their ids in ascending order, 4 bits each
+  u32 epar = 0, ecpar = 0;    // base full / comp phase parity per ring position
+  u32 li = 0, lu = 0;         // ring position / use parity of the next load
+  bool wanting = false, shrink = false;
+  u32 published = 0;          // tiles announced to the combine warps
+  u32 ebase = 0;              // first tile of the epoch
+  const u32 want_self = Lwant + 4 * (Lbar - 1), want_other = Lwant + 4 * (2 - Lbar);
+#endif
   int sj = 0;                 // store cursor
   u32 st = 0;
   int pj = 0;                 // next micro-batch to post
   i64 lo_l = 0, nb_l = 0, lo_s = 0, nb_s = 0, lo_p = 0, nb_p = 0;
-  u32 T_l = mb_tiles<F>(a, p.len, 0, L.inst, T::kSize, lo_l, nb_l);
+  u32 T_l = mb_tiles_m<F>(aM, aMi, plen, 0, Linst, T::kSize, lo_l, nb_l);
   u32 T_s = T_l;
   lo_s = lo_l;
   nb_s = nb_l;
@@ -767,7 +844,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       while (wp < nmb) {
         bool ok = true;
         for (int k = 0; k < d.ndeps && ok; ++k)
-          ok = ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) >= dep_target(a, d, k, wp);
+          ok = ready_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, wp));
         if (!ok) break;
         post_writable<F>(a, d, p, wp);
         ++wp;
@@ -776,11 +853,11 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
     }
 #if RESCCL_PREFETCH
     // (0) keep the local operand of the next RESCCL_PREFETCH micro-batches streaming into L2
-    if (p.A && (F & (kReduce | kRecv)) != kRecv) {
+    if (pA && (F & (kReduce | kRecv)) != kRecv) {
       while (pf < nmb && pf <= lj + RESCCL_PREFETCH) {
         i64 lo_f, nb_f;
-        mb_tiles<F>(a, p.len, pf, L.inst, T::kSize, lo_f, nb_f);
-        if (nb_f > 0) l2_prefetch(p.A + lo_f * T::kSize, (u32)nb_f);
+        mb_tiles_m<F>(aM, aMi, plen, pf, Linst, T::kSize, lo_f, nb_f);
+        if (nb_f > 0) l2_prefetch(pA + lo_f * T::kSize, (u32)nb_f);
         ++pf;
       }
     }
@@ -796,84 +873,135 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       if (lt >= T_l) {
         ++lj;
         lt = 0;
-        if (lj < nmb) T_l = mb_tiles<F>(a, p.len, lj, L.inst, T::kSize, lo_l, nb_l);
+        if (lj < nmb) T_l = mb_tiles_m<F>(aM, aMi, plen, lj, Linst, T::kSize, lo_l, nb_l);
         continue;
       }
-      int sc = (issued - released < (u32)RESCCL_POOL_CAP) ? pool_claim(L.pool) : -1;
-      if (sc < 0 && stored > released) {  // recycle our oldest stored stage (its store read it out)
-        const u32 keep = stored - released - 1 < 15 ? stored - released - 1 : 15;
-        tma_wait_read_n(keep);
-        const u32 upto = stored - keep;
-        for (; released < upto; ++released) pool_release(L.pool, RESCCL_HS(released % P));
-        if (issued - released < (u32)RESCCL_POOL_CAP) sc = pool_claim(L.pool);
+#if !RESCCL_RING
+      if (shrink) break;
+      if (eR == 0) {  // start an epoch: take the free stages
+        u32 m = atoms_and(Lpool, 0u);
+        const u32 cap = lds_u32(want_other) ? (P / 2 < RESCCL_POOL_CAP ? P / 2 : RESCCL_POOL_CAP)
+                                            : (u32)RESCCL_POOL_CAP;
+        u32 keep = 0;
+        for (u32 n = 0; m && n < cap; ++n) {
+          const u32 b = m & (0u - m);
+          keep |= b;
+          m &= ~b;
+        }
+        if (m) atoms_or(Lpool, m);  // over the cap: give back
+        if (!keep) {
+          if (!wanting) sts_u32(want_self, 1u);
+          wanting = true;
+          break;  // the other lane holds the pool: its tiles drain by themselves
+        }
+        if (wanting) sts_u32(want_self, 0u);
+        wanting = false;
+        emask = keep;
+        eR = (u32)__popc(keep);
+        ering = 0;
+        epar = 0;
+        ecpar = 0;
+        for (u32 i = 0, mm = keep; mm; ++i) {
+          const u32 s = (u32)(__ffs(mm) - 1);
+          mm &= mm - 1;
+          ering |= (u64)s << (4 * i);
+          epar |= mbar_phase(Lfull + 8 * s) << i;
+          ecpar |= mbar_phase(Lcomp + 8 * s) << i;
+        }
+        li = 0;
+        lu = 0;
+        ebase = k0 + issued;
+        // the combine warps map this epoch's tiles through (first tile, stages, parities);
+        // the announcements carry the first tile too, so a reader validates the
+        // descriptor against them (no fence)
+        if (F & kReduce) sts_u64(Lqdesc, (u64)ebase | ((u64)emask << 32) | ((u64)epar << 48));
       }
-      if (sc < 0) break;  // the other lane holds the pool: its tiles drain by themselves
-      const u32 s = (u32)sc;
+#endif
+      if (issued - released >= eR) {  // the tile eR back still holds the stage we need next
+        if (stored > released && (stored - released >= (u32)RESCCL_STORE_LAG || issued == stored)) {
+          const u32 keep = stored - released - 1 < 15 ? stored - released - 1 : 15;
+          tma_wait_read_n(keep);
+          released = stored - keep;
+        }
+        if (issued - released >= eR) break;
+      }
       const u32 k = k0 + issued;
       const u32 slot = issued % P;
-      const u32 fu = lds_u32(L.fuse + 4 * s);
-      const u32 fpar = fu & 1;
+#if RESCCL_RING
+      const u32 s = Lring0 + k % RESCCL_TMA_STAGES;
+      const u32 fpar = (k / RESCCL_TMA_STAGES) & 1;
+      if (F & kReduce) {
+        const u32 rb = 1u << (k % RESCCL_TMA_STAGES);
+        hc = (hc & ~(1u << slot)) | (((Lcpar & rb) ? 1u : 0u) << slot);
+        Lcpar ^= rb;
+      }
+#else
+      const u32 s = (u32)(ering >> (4 * li)) & 15u;
+      const u32 fpar = ((epar >> li) & 1u) ^ lu;
+      if (F & kReduce) hc = (hc & ~(1u << slot)) | ((((ecpar >> li) & 1u) ^ lu) << slot);
+      if (++li == eR) {
+        li = 0;
+        lu ^= 1u;
+      }
+      // every 32 tiles: the other lane waits for stages while we hold more than half
+      if (eR > P / 2 && (issued & 31) == 31 && lds_u32(want_other)) shrink = true;
+#endif
       hs = (hs & ~(15ull << (4 * slot))) | ((u64)s << (4 * slot));
       hf = (hf & ~(1u << slot)) | (fpar << slot);
-      sts_u32(L.fuse + 4 * s, fu + 1);
-      if (F & kReduce) {
-        const u32 cu = lds_u32(L.cuse + 4 * s);
-        hc = (hc & ~(1u << slot)) | ((cu & 1) << slot);
-        sts_u32(L.cuse + 4 * s, cu + 1);
-        sts_u8(L.qst + k % RESCCL_QN, s);
-        sts_u8(L.qpar + k % RESCCL_QN, fpar);
-      }
       const i64 off = (i64)lt * TB;
       const u32 nb = (u32)((nb_l - off) < TB ? (nb_l - off) : TB);
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
       if (F & kReduce) {
         const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + lj;
-        const char* bsrc = (F & kDirect) ? p.R + lo_l * T::kSize + off
-                                         : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off;
-        mbar_expect_tx(L.full + 8 * s, 2 * nb);
-        tma_load(sa, p.A + lo_l * T::kSize + off, nb, L.full + 8 * s, pol_first);
-        tma_load(sa + (u32)RESCCL_TMA_TILE, bsrc, nb, L.full + 8 * s, pol_first);
+        const char* bsrc = (F & kDirect) ? pR + lo_l * T::kSize + off
+                                         : pin + (in_seq % RESCCL_K) * RESCCL_SLOT + off;
+        mbar_expect_tx(Lfull + 8 * s, 2 * nb);
+        tma_load(sa, pA + lo_l * T::kSize + off, nb, Lfull + 8 * s, pol_first);
+        tma_load(sa + (u32)RESCCL_TMA_TILE, bsrc, nb, Lfull + 8 * s, pol_first);
       } else {
         const char* src;
         if (Kind<F>::has_b) {  // staged receive: the FIFO slot
           const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + lj;
-          src = p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + off;
+          src = pin + (in_seq % RESCCL_K) * RESCCL_SLOT + off;
         } else {               // send / pushed payload forwarded: our location
-          src = p.A + lo_l * T::kSize + off;
+          src = pA + lo_l * T::kSize + off;
         }
-        mbar_expect_tx(L.full + 8 * s, nb);
-        tma_load(sa, src, nb, L.full + 8 * s, pol_first);
+        mbar_expect_tx(Lfull + 8 * s, nb);
+        tma_load(sa, src, nb, Lfull + 8 * s, pol_first);
       }
+      (void)k;
       ++issued;
       ++lt;
-      if (F & kReduce) {
-        fence_cta();  // qst / qpar before the issued count
-        sts_u32(L.issued, k0 + issued);
-      }
       prog = true;
     }
+#if !RESCCL_RING
+    if ((F & kReduce) && published != issued) {  // one word per batch of issued tiles
+      sts_u64(Lqprog, ((u64)ebase << 32) | (u64)(k0 + issued));
+      published = issued;
+    }
+#endif
     // (3) stores
     while (stored < issued) {
       const u32 slot = stored % P;
       const u32 s = RESCCL_HS(slot);
-      const bool ok = (F & kReduce) ? mbar_test(L.comp + 8 * s, (hc >> slot) & 1)
-                                    : mbar_test(L.full + 8 * s, (hf >> slot) & 1);
+      const bool ok = (F & kReduce) ? mbar_test(Lcomp + 8 * s, (hc >> slot) & 1)
+                                    : mbar_test(Lfull + 8 * s, (hf >> slot) & 1);
       if (!ok) break;
       while (st >= T_s) {
         ++sj;
         st = 0;
-        T_s = mb_tiles<F>(a, p.len, sj, L.inst, T::kSize, lo_s, nb_s);
+        T_s = mb_tiles_m<F>(aM, aMi, plen, sj, Linst, T::kSize, lo_s, nb_s);
       }
       const i64 off = (i64)st * TB;
       const u32 nb = (u32)((nb_s - off) < TB ? (nb_s - off) : TB);
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
-      if (F & kStore) tma_store(p.D1 + lo_s * T::kSize + off, sa, nb, pol_first);
+      if (F & kStore) tma_store(pD1 + lo_s * T::kSize + off, sa, nb, pol_first);
       if (Kind<F>::send_data) {
         if (F & kDirect) {
-          tma_store(p.Q + lo_s * T::kSize + off, sa, nb, pol_first);
+          tma_store(pQ + lo_s * T::kSize + off, sa, nb, pol_first);
         } else {
           const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + sj;
-          tma_store(p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + off, sa, nb, pol_last);
+          tma_store(pout + (out_seq % RESCCL_K) * RESCCL_SLOT + off, sa, nb, pol_last);
         }
       }
       tma_commit();
@@ -884,33 +1012,47 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
     // (4) post
     if (pj < rj && stored >= gp_end) {
       tma_wait_n(stored - gp_end);
-      for (; released < gp_end; ++released) pool_release(L.pool, RESCCL_HS(released % P));  // written out
+      if (released < gp_end) released = gp_end;  // written out
       // unaligned tail (< 16 bytes) of this micro-batch: scalar, by the leader
       i64 lo_h, hi_h;
-      slice_of(a, p.len, pj, L.inst, lo_h, hi_h);
+      slice_of_m(aM, aMi, plen, pj, Linst, lo_h, hi_h);
       const i64 e0 = lo_h + nb_p / T::kSize;
       if (e0 < hi_h) {
         const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + pj;
         const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + pj;
-        const char* Bj = Kind<F>::has_b ? ((F & kDirect) ? p.R + e0 * T::kSize
-                                                         : p.in_data + (in_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
+        const char* Bj = Kind<F>::has_b ? ((F & kDirect) ? pR + e0 * T::kSize
+                                                         : pin + (in_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
                                         : nullptr;
-        char* D2j = Kind<F>::send_data ? ((F & kDirect) ? p.Q + e0 * T::kSize
-                                                        : p.out_data + (out_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
+        char* D2j = Kind<F>::send_data ? ((F & kDirect) ? pQ + e0 * T::kSize
+                                                        : pout + (out_seq % RESCCL_K) * RESCCL_SLOT + nb_p)
                                        : nullptr;
         for (i64 e = 0; e < hi_h - e0; ++e)
-          elem_move<T, OP>(Kind<F>::mf, p.A ? p.A + e0 * T::kSize : nullptr, Bj,
-                           p.D1 ? p.D1 + e0 * T::kSize : nullptr, D2j, e);
+          elem_move<T, OP>(Kind<F>::mf, pA ? pA + e0 * T::kSize : nullptr, Bj,
+                           pD1 ? pD1 + e0 * T::kSize : nullptr, D2j, e);
       }
       fence_proxy_async();
       post_mb<F>(a, d, p, pj);
       ++pj;
       if (pj < nmb) {
-        T_p = mb_tiles<F>(a, p.len, pj, L.inst, T::kSize, lo_p, nb_p);
+        T_p = mb_tiles_m<F>(aM, aMi, plen, pj, Linst, T::kSize, lo_p, nb_p);
         gp_end += T_p;
       }
       prog = true;
     }
+#if !RESCCL_RING
+    // (5) end the epoch once everything loaded is stored and no ready work is left (or
+    // when shrinking), after the stores have read their stages out
+    if (eR && stored == issued && (lj == rj || shrink)) {
+      if (stored > released) {
+        tma_wait_read_n(0);
+        released = stored;
+      }
+      atoms_or(Lpool, emask);
+      eR = 0;
+      emask = 0;
+      shrink = false;
+    }
+#endif
     if (prog) {
 #if RESCCL_TRACE
       if (t_idle) L.wait_ns += globaltimer() - t_idle;
@@ -921,7 +1063,17 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
 #if RESCCL_TRACE
       if (t_idle == 0) t_idle = globaltimer();
 #endif
-      if (++spins > 32) nanosleep_(20);
+      if (stored < issued) {
+        // idle with a tile outstanding: sleep on the oldest one's barrier (it is the next
+        // event the store step needs) instead of polling
+        const u32 slot = stored % P;
+        const u32 s = RESCCL_HS(slot);
+        if (F & kReduce) (void)mbar_try(Lcomp + 8 * s, (hc >> slot) & 1);
+        else (void)mbar_try(Lfull + 8 * s, (hf >> slot) & 1);
+        ++spins;
+      } else if (++spins > 32) {
+        nanosleep_(20);
+      }
       if ((spins & 255) == 0) {
         const u64 now = globaltimer();
         if (t_idle == 0) t_idle = now;
@@ -935,13 +1087,18 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   }
   if (stored > released) {  // (all posted: every store has completed)
     tma_wait_read_n(0);
-    for (; released < stored; ++released) pool_release(L.pool, RESCCL_HS(released % P));
+    released = stored;
   }
+#if !RESCCL_RING
+  if (eR) atoms_or(Lpool, emask);
+  if (wanting) sts_u32(want_self, 0u);
+#endif
 #undef RESCCL_HS
 #if RESCCL_TRACE
   if (t_idle) L.wait_ns += globaltimer() - t_idle;
 #endif
   L.tseq = k0 + issued;
+  L.cpar = Lcpar;
   return true;
 }
 
@@ -951,31 +1108,63 @@ template <class T, int OP, int F>
 __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const PrimPtrs& p, int ctid, int nct) {
   const KArgs& a = *L.a;
   const i64 TB = RESCCL_TMA_TILE;  // reduce tiles only
+  const u32 Lfull = L.full, Lcomp = L.comp, Lstage = L.stage, Lqprog = L.qprog, Lqdesc = L.qdesc, Lring0 = L.ring0;
+  const int Linst = L.inst, nmb = a.n_mb;
+  const i64 aM = a.M, aMi = a.Mi, plen = p.len;
+  volatile int* const abort_flag = L.abort_flag;
   u32 k = L.tseq;
-  for (int j = 0; j < a.n_mb; ++j) {
+#if !RESCCL_RING
+  u32 cbase = 0xFFFFFFFFu, cmask = 0, cpar = 0, cR = 1, ci = 0, cu = 0;  // cached epoch, position of k
+#endif
+  for (int j = 0; j < nmb; ++j) {
     i64 lo, nbj;
-    const u32 ntl = mb_tiles<F>(a, p.len, j, L.inst, T::kSize, lo, nbj);
+    const u32 ntl = mb_tiles_m<F>(aM, aMi, plen, j, Linst, T::kSize, lo, nbj);
     for (u32 t = 0; t < ntl; ++t, ++k) {
       const i64 off = (i64)t * TB;
       const int nb = (int)((nbj - off) < TB ? (nbj - off) : TB);
       u32 spins = 0;
-      while ((int)(lds_u32(L.issued) - k) <= 0) {  // tile k not issued yet
+#if RESCCL_RING
+      // stage and phase follow from k (the leader cannot re-arm the stage for tile k + S
+      // before every combine warp arrived for tile k: no parity ABA)
+      const u32 s = Lring0 + k % RESCCL_TMA_STAGES;
+      const u32 par = (k / RESCCL_TMA_STAGES) & 1;
+#else
+      // wait until the leader announced tile k (announcement = epoch's first tile << 32 |
+      // tiles issued), then map it through that epoch: the epoch holding tile k cannot end
+      // before this warp combined it, so the announcing epoch is k's
+      u64 w;
+      while ((int)((u32)(w = lds_u64(Lqprog)) - k) <= 0) {
         if (++spins > 16) nanosleep_(20);
-        if ((spins & 1023) == 0 && *L.abort_flag) return false;
+        if ((spins & 1023) == 0 && *abort_flag) return false;
       }
-      fence_cta();
-      const u32 s = lds_u8(L.qst + k % RESCCL_QN);
-      const u32 par = lds_u8(L.qpar + k % RESCCL_QN);
-      while (!mbar_test(L.full + 8 * s, par)) {
-        if (++spins > 16) nanosleep_(20);
-        if ((spins & 1023) == 0 && *L.abort_flag) return false;
+      const u32 eb = (u32)(w >> 32);
+      if (eb != cbase) {  // a new epoch: its descriptor (validated by its first tile)
+        u64 dsc;
+        while ((u32)(dsc = lds_u64(Lqdesc)) != eb) {
+        }
+        cbase = eb;
+        cmask = (u32)(dsc >> 32) & 0xFFFFu;
+        cpar = (u32)(dsc >> 48);
+        cR = (u32)__popc(cmask);
+        ci = (k - eb) % cR;
+        cu = ((k - eb) / cR) & 1u;
       }
-      const u32 sa = L.stage + s * 2 * (u32)TB;
-      for (int i = ctid; i < nb / 16; i += nct)
-        sts_v4(sa + 16 * i, combine_v<T, OP>(lds_v4(sa + 16 * i), lds_v4(sa + (u32)TB + 16 * i)));
+      const u32 s = nth_bit(cmask, ci);
+      const u32 par = ((cpar >> ci) & 1u) ^ cu;
+      if (++ci == cR) {
+        ci = 0;
+        cu ^= 1u;
+      }
+#endif
+      while (!mbar_try(Lfull + 8 * s, par)) {  // (stage s is held for tile k: no parity ABA)
+        if ((++spins & 63) == 0 && *abort_flag) return false;
+      }
+      const u32 sa = Lstage + s * 2 * (u32)TB;
+      for (int i2 = ctid; i2 < nb / 16; i2 += nct)
+        sts_v4(sa + 16 * i2, combine_v<T, OP>(lds_v4(sa + 16 * i2), lds_v4(sa + (u32)TB + 16 * i2)));
       fence_proxy_async_smem();
       __syncwarp();
-      if ((threadIdx.x & 31) == 0) mbar_arrive(L.comp + 8 * s);
+      if ((threadIdx.x & 31) == 0) mbar_arrive(Lcomp + 8 * s);
     }
   }
   L.tseq = k;
@@ -1001,7 +1190,7 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
     if (wp < nmb) {
       bool ok = true;
       for (int k = 0; k < d.ndeps && ok; ++k)
-        ok = ld_acquire(at(L.self, d.deps[k] + (i64)L.inst * 128)) >= dep_target(a, d, k, wp);
+        ok = ready_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, wp));
       if (ok) {
         fence_release();
         if (!recv) {
@@ -1017,7 +1206,7 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
     }
     if (recv && dj < wp) {
       const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + dj;
-      if (ld_acquire(p.in_flag + (in_seq % RESCCL_K)) >= in_seq + 1) {
+      if (ready_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1)) {
         fence_release();
         if (F & kSend) {  // drecv_p: the payload is in our location -> readable for the next hop
           const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + dj;
@@ -1131,7 +1320,7 @@ __device__ __noinline__ void exit_barrier(const KArgs& a, int rank, int nranks, 
     if (q == rank) continue;
     const u64 target = (a.epoch + 1) * (u64)blocks[q];
     u32 spins = 0;
-    while (ld_acquire(at(a.arena[q], off)) < target) {
+    while (!ready_ge(at(a.arena[q], off), target)) {
       if (++spins > 64) nanosleep_(64);
       if ((spins & 1023) == 0 && globaltimer() - t0 > a.timeout_ns) {
         atomicCAS(a.err, 0, kErrTimeout);

@@ -58,6 +58,8 @@ struct CodegenOpts {
   int jitter = 0;                // debug fault injector: random delays around every sync
   int prefetch = 0;              // micro-batches of local operand prefetched into L2 ahead (off: r01)
   int pool_cap = 0;              // stages of the CTA pool one lane may hold (0 = all)
+  int ring = 0;                  // lane-private stage rings instead of the shared CTA pool
+  int store_lag = 1;             // bulk stores a lane lets drain before it blocks to reuse a stage
   int exit_barrier = 0;          // direct transport across processes: a rank's kernel ends only
                                  // after every peer's blocks finished touching its buffers
 };

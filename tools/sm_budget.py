@@ -5,7 +5,7 @@ bytes) and the SMs the launch occupies.
 
   python tools/sm_budget.py [S_MiB] [geometry ...]
 geometry: "two" = 256-thread CTAs, 2 x 12 KiB-tile stages (two CTAs per SM);
-          "one" = 512-thread CTAs, 4 x 16 KiB-tile stages (one CTA per SM)."""
+          "one" = 512-thread CTAs, 4 x 12 KiB-tile stages (one CTA per SM)."""
 import json
 import os
 import sys
@@ -17,23 +17,28 @@ import paper_conf_sigcomm_liuhlgcwz025_b200 as R
 N = 8
 S = int(float(sys.argv[1]) * (1 << 20)) if len(sys.argv) > 1 else 256 << 20
 GEOS = sys.argv[2:] or ["two", "one"]
-GEO = {"two": dict(nwarps=8, tmastages=2, tmatile=12288), "one": dict(nwarps=16, tmastages=4, tmatile=16384)}
+GEO = {"two": dict(nwarps=8, tmastages=2, tmatile=12288), "one": dict(nwarps=16, tmastages=4, tmatile=12288)}
 EXTRA = os.environ.get("SMB_OPTS", "")
+COLL = os.environ.get("SMB_COLL", "allreduce")
 INST = [int(x) for x in os.environ.get("SMB_INST", "1,2,3,4,6,8,10,12,16,18,24,30,37").split(",")]
 n_sm = torch.cuda.get_device_properties(0).multi_processor_count
 
-cnt = S // 2
-s = [(torch.rand(cnt, device="cuda:0") * 2 - 1).to(torch.bfloat16) for _ in range(N)]
-r = [torch.empty_like(x) for x in s]
+cnt = S // 2  # AR: count; AG: total output; RS: total input (nccl-tests S)
+sn, rn = {"allreduce": (cnt, cnt), "allgather": (cnt // N, cnt), "reducescatter": (cnt, cnt // N)}[COLL]
+s = [(torch.rand(sn, device="cuda:0") * 2 - 1).to(torch.bfloat16) for _ in range(N)]
+r = [torch.empty(rn, device="cuda:0", dtype=torch.bfloat16) for _ in range(N)]
+# algorithmic HBM bytes per rank (direct transport): AR 5(N-1)/N S, RS 3(N-1)/N S, AG 2(N-1)/N S
+HB = {"allreduce": 5.0, "reducescatter": 3.0, "allgather": 2.0}[COLL]
+BUSF = {"allreduce": 2.0 * (N - 1) / N}.get(COLL, (N - 1) / N)
 for geo in GEOS:
     for inst in INST:
         if geo == "one" and inst * N > n_sm:
             continue
         if inst * N > 2 * n_sm:
             continue
-        cb = max(1 << 20, min(32 << 20, S // N))
+        cb = int(os.environ.get("SMB_CB", max(1 << 20, min(32 << 20, S // N))))
         opts = dict(instances=inst, chunkbytes=cb, fifodepth=2, direct=1, **GEO[geo])
-        text = R.rescclGenerateIr("ring", "allreduce", N)
+        text = R.rescclGenerateIr("ring", COLL, N)
         h, rest = text.split("\n", 1)
         h += "".join(f" {k}={v}" for k, v in opts.items()) + (" " + EXTRA if EXTRA else "")
         grp = R.VirtualGroup(N, 0)
@@ -41,20 +46,20 @@ for geo in GEOS:
             grp.load(h + "\n" + rest)
             info = grp.plan_info()
             for _ in range(3):
-                grp.allreduce(s, r)
+                getattr(grp, COLL)(s, r)
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             it = 10
             e0.record()
             for _ in range(it):
-                grp.allreduce(s, r)
+                getattr(grp, COLL)(s, r)
             e1.record()
             torch.cuda.synchronize()
             ms = e0.elapsed_time(e1) / it
             blocks = sum(info["blocks_per_rank"])
-            bus = S / (ms * 1e-3) / 1e9 * 2 * (N - 1) / N
-            hbm = 5.0 * (N - 1) / N * S * N / (ms * 1e-3) / 1e9
-            print(json.dumps({"geometry": geo, "instances": inst, "ctas": blocks,
+            bus = S / (ms * 1e-3) / 1e9 * BUSF
+            hbm = HB * (N - 1) / N * S * N / (ms * 1e-3) / 1e9
+            print(json.dumps({"coll": COLL, "geometry": geo, "instances": inst, "ctas": blocks,
                               "sms": min(n_sm, blocks),
                               "S": S, "us": round(ms * 1e3, 1), "busbw_gbs": round(bus, 1),
                               "hbm_gbs": round(hbm, 1), "per_sm_hbm_gbs": round(hbm / min(n_sm, blocks), 1),
