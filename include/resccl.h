@@ -166,6 +166,42 @@ rescclResult_t rescclAllGather(const void* sendbuf, void* recvbuf, size_t sendco
 rescclResult_t rescclReduceScatter(const void* sendbuf, void* recvbuf, size_t recvcount,
                                    rescclDataType_t dtype, rescclRedOp_t op, rescclComm_t comm, void* stream);
 
+/* ------------------------------------------------------------------ f3: NVLS (NVLink SHARP) windows */
+
+/* not in the paper: the NVSwitch-SHARP transport variant.  An NVLS
+ * window is `bytes` of device memory on every rank, all bound into one multicast object,
+ * so that multimem.ld_reduce through the multicast alias returns the switch-computed
+ * reduction of every rank's copy and multimem.st lands in every rank's copy.  An
+ * algorithm loaded with the header option nvls=1 (env RESCCL_NVLS=1; CTAs per rank:
+ * nvlsctas=16) runs a call on the NVLS kernel when
+ *   - its send and receive buffers lie in NVLS windows at 4-byte-aligned offsets, the
+ *     same on every rank (allocate windows in the same order and size everywhere),
+ *   - each rank's block (AR: the buffer; RS: recvcount; AG: sendcount) is a whole number
+ *     of 4-byte granules (2-byte dtypes: even counts), and
+ *   - the op has a multimem form (all but float32 max/min);
+ * otherwise the algorithm's primitive plan runs.  The NVLS schedule on the collective's
+ * chunk layout: ReduceScatter mred(r): <r,r> := (+)_k <k,r>; AllGather mcast(r):
+ * <k,r> := <r,r> for all k; AllReduce = mred + mcast of 16-byte-aligned slices
+ * (reading R28).  bf16/fp16 sums accumulate in fp32 inside the switch.
+ * Windows are owned by the communicator (freed by rescclNvlsFree or rescclCommDestroy);
+ * the returned pointer is the window's first byte (4 KiB aligned).
+ * CudaError when the driver or the fabric refuses multicast (message names the call and
+ * the failing rank); every rank of a multi-process allocation returns it. */
+
+/* *supported = CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED of the communicator's device
+ * (0 for virtual ranks, which share one device). */
+rescclResult_t rescclNvlsSupported(rescclComm_t comm, int* supported);
+/* Multi-process, collective over all ranks: rank 0 creates the multicast object and
+ * exports a fabric handle, the `allgather` callback (as for rescclCommInit) carries it
+ * and two status rounds; every rank makes the same three callback calls even when a
+ * step fails locally, so a failure anywhere returns an error everywhere. */
+rescclResult_t rescclNvlsAlloc(rescclComm_t comm, size_t bytes, int (*allgather)(const void* in, void* out, size_t len, void* ctx),
+                               void* ctx, void** ptr);
+/* Single process, one device per rank (rescclCommInitAll with distinct devices):
+ * comms[k] is rank k of n; ptrs[k] receives rank k's window. */
+rescclResult_t rescclNvlsAllocAll(rescclComm_t* comms, int n, size_t bytes, void** ptrs);
+rescclResult_t rescclNvlsFree(rescclComm_t comm, void* ptr);
+
 /* ------------------------------------------------------------------ host-only tools (no GPU needed) */
 
 /* Built-in generators (name in ring|dbt|hm|synth; opts "g=4 seed=0 fanout=2").
@@ -191,6 +227,9 @@ rescclResult_t rescclCodegenIr(const char* irText, const char* opts, int rank_lo
  * receives the cubin size. */
 rescclResult_t rescclCompileIr(const char* irText, const char* opts, rescclDataType_t dtype, rescclRedOp_t op,
                                size_t* cubin_bytes);
+/* NVRTC-compile the NVLS kernel of a collective for sm_100a (no GPU needed); InvalidArgument
+ * for a bad coll/dtype/op.  (float32 max/min compile but are never launched.) */
+rescclResult_t rescclCompileNvls(rescclColl_t coll, rescclDataType_t dtype, rescclRedOp_t op, size_t* cubin_bytes);
 /* Control-only blocking simulation of a planned IR (invariant I4): *ok = 1 if the
  * plan completes for FIFO depth K and n_mb micro-batches. */
 rescclResult_t rescclCheckDeadlock(const char* irText, const char* opts, int K, int n_mb, int* ok);

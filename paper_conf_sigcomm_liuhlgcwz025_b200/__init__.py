@@ -47,6 +47,7 @@ EXPORTS = [
     "rescclAllGather", "rescclReduceScatter", "rescclGenerateIr", "rescclPlanIr",
     "rescclCodegenIr", "rescclCompileIr", "rescclCheckDeadlock", "rescclParseResCCLang", "rescclProfilePlanner",
     "rescclCommRegister", "rescclCommRegisterConnect", "rescclSimulateTimeline",
+    "rescclNvlsSupported", "rescclNvlsAlloc", "rescclNvlsAllocAll", "rescclNvlsFree", "rescclCompileNvls",
 ]
 
 _c = ctypes
@@ -80,6 +81,11 @@ _SIGS = {
     "rescclProfilePlanner": (_i, [_c.c_char_p, _c.c_char_p, _i, _c.c_char_p, _c.POINTER(_sz)]),
     "rescclCommRegister": (_i, [_vp, _vp, _sz, _vp, _c.POINTER(_sz)]),
     "rescclCommRegisterConnect": (_i, [_vp, _c.POINTER(_vp), _c.POINTER(_sz), _c.POINTER(_i)]),
+    "rescclNvlsSupported": (_i, [_vp, _c.POINTER(_i)]),
+    "rescclNvlsAlloc": (_i, [_vp, _sz, _vp, _vp, _c.POINTER(_vp)]),
+    "rescclNvlsAllocAll": (_i, [_c.POINTER(_vp), _i, _sz, _c.POINTER(_vp)]),
+    "rescclNvlsFree": (_i, [_vp, _vp]),
+    "rescclCompileNvls": (_i, [_i, _i, _i, _c.POINTER(_sz)]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -176,6 +182,51 @@ def rescclCommRegisterConnect(comm: int, blobs: Sequence[bytes]) -> int:
     w = _i()
     _check(_lib.rescclCommRegisterConnect(comm, arr, lens, _c.byref(w)), "rescclCommRegisterConnect")
     return w.value
+
+
+# allgather callback of rescclCommInit / rescclNvlsAlloc: int (*)(const void*, void*, size_t, void*)
+ALLGATHER_CB = _c.CFUNCTYPE(_i, _vp, _vp, _sz, _vp)
+
+
+def rescclNvlsSupported(comm: int) -> bool:
+    v = _i()
+    _check(_lib.rescclNvlsSupported(comm, _c.byref(v)), "rescclNvlsSupported")
+    return bool(v.value)
+
+
+def rescclNvlsAlloc(comm: int, nbytes: int, allgather) -> int:
+    """Multi-process NVLS window (collective).  `allgather(data: bytes) -> List[bytes]`
+    gathers one equal-length blob from every rank, rank-major."""
+    def cb(inp, out, n, _ctx):
+        try:
+            parts = allgather(_c.string_at(inp, n))
+            joined = b"".join(parts)
+            _c.memmove(out, joined, len(joined))
+            return 0
+        except Exception:  # noqa: BLE001 -- reported through the C ABI as a SystemError
+            return 1
+    fn = ALLGATHER_CB(cb)
+    p = _vp()
+    _check(_lib.rescclNvlsAlloc(comm, nbytes, _c.cast(fn, _vp), None, _c.byref(p)), "rescclNvlsAlloc")
+    return p.value
+
+
+def rescclNvlsAllocAll(comms: Sequence[int], nbytes: int) -> List[int]:
+    n = len(comms)
+    arr = (_vp * n)(*comms)
+    ptrs = (_vp * n)()
+    _check(_lib.rescclNvlsAllocAll(arr, n, nbytes, ptrs), "rescclNvlsAllocAll")
+    return [ptrs[k] for k in range(n)]
+
+
+def rescclNvlsFree(comm: int, ptr: int) -> None:
+    _check(_lib.rescclNvlsFree(comm, ptr), "rescclNvlsFree")
+
+
+def rescclCompileNvls(coll: str, dtype: str = "bfloat16", op: str = "sum") -> int:
+    n = _sz(0)
+    _check(_lib.rescclCompileNvls(COLLS[coll], DTYPES[dtype], OPS[op], _c.byref(n)), "rescclCompileNvls")
+    return n.value
 
 
 def rescclCommDestroy(comm: int) -> None:

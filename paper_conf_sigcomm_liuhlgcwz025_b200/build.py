@@ -110,6 +110,15 @@ def selftest_cubin() -> str:
     _run([NVCC, "-cubin", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
           "-I", os.path.join(CSRC, "device"), "-DRESCCL_T=rdev::TBF16", "-DRESCCL_OP=0", "-Xptxas", "-v",
           cu, "-o", cubin])
+    # f3: the NVLS kernel (multimem.ld_reduce / multimem.st), bf16 sum AllReduce
+    nv = os.path.join(BUILD, "selftest_nvls_ar.cu")
+    with open(nv, "w") as f:
+        f.write('#include "resccl_device.cuh"\n'
+                'extern "C" __global__ void __launch_bounds__(512, 1) resccl_nvls_kernel(rdev::NvlsArgs a) {\n'
+                '  rdev::nvls_run<RESCCL_T, RESCCL_OP, 2>(a);\n}\n')
+    _run([NVCC, "-cubin", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
+          "-I", os.path.join(CSRC, "device"), "-DRESCCL_T=rdev::TBF16", "-DRESCCL_OP=0", "-Xptxas", "-v",
+          nv, "-o", os.path.join(BUILD, "selftest_nvls_ar.cubin")])
     return cubin
 
 

@@ -146,6 +146,8 @@ struct Options {
   int ring = 0;      // lane-private TMA stage rings (1) vs one pool shared by both lanes (0)
   int store_lag = 1; // bulk stores a lane lets drain before it blocks to reuse a stage
   int sys_rank = -1; // rescclCompileIr / rescclCodegenIr: one rank's multi-process (.sys) kernel
+  int nvls = 0;      // f3: NVLS transport for calls whose buffers lie in NVLS windows
+  int nvls_ctas = 16;  // CTAs (x 512 threads) per rank of an NVLS launch
 };
 
 std::map<std::string, std::string> parse_kv(const char* s) {
@@ -193,6 +195,8 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "poolcap") o.pool_cap = (int)to_long(v, k);
   else if (k == "storelag") o.store_lag = (int)to_long(v, k);
   else if (k == "ring") o.ring = (int)to_long(v, k);
+  else if (k == "nvls") o.nvls = (int)to_long(v, k);
+  else if (k == "nvlsctas") o.nvls_ctas = (int)to_long(v, k);
   else if (k == "sched") {
     if (v == "hpds") o.sched = 0;
     else if (v == "rr") o.sched = 1;
@@ -213,7 +217,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -224,6 +228,7 @@ Options make_options(const Ir& ir, const char* extra) {
   if (o.tma_tile < 1024 || o.tma_tile % 128 || o.tma_stages < 1 || o.tma_stages > 8 ||
       4 * o.tma_tile * o.tma_stages > 200 * 1024)
     fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 4*tile*stages <= 200 KiB");
+  if (o.nvls_ctas < 1 || o.nvls_ctas > 148) fail(rescclInvalidArgument, "nvlsctas must be 1..148");
   if (o.store_lag < 1 || o.store_lag > o.tma_stages)
     fail(rescclInvalidArgument, "storelag must be 1..tmastages");
   return o;
@@ -354,6 +359,7 @@ struct rescclAlgo {
 
 namespace {
 struct Group;
+struct NvlsWin;
 }
 
 struct rescclComm {
@@ -381,6 +387,7 @@ struct rescclComm {
   };
   std::vector<Window> windows;
   std::map<std::string, char*> ipc_maps;  // opened peer allocations (handle bytes -> mapped base)
+  std::vector<std::shared_ptr<NvlsWin>> nvls;  // f3: this rank's NVLS windows (multicast-bound)
 };
 
 namespace {
@@ -462,7 +469,7 @@ std::string info_json(const AlgoShared& a) {
   o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
     << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"tma\":" << a.opt.tma
     << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"l2hint\":" << a.opt.l2hint << ",\"prefetch\":" << a.opt.prefetch << ",\"sched\":\""
-    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"linkmodel\":\""
+    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"nvls\":" << a.opt.nvls << ",\"nvlsctas\":" << a.opt.nvls_ctas << ",\"linkmodel\":\""
     << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
     << ",\"ctas\":[";
   for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];
@@ -739,6 +746,8 @@ void group_launch(Group* G, Pending& p) {
 }
 
 rescclAlgo* ensure_algo(rescclComm* comm, Coll coll);
+bool try_nvls(rescclComm* comm, const AlgoShared& a, int coll, const void* send, void* recv, size_t count,
+              rescclDataType_t dt, rescclRedOp_t op, cudaStream_t s);
 
 void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t count, rescclDataType_t dt,
                 rescclRedOp_t op, void* stream) {
@@ -751,6 +760,7 @@ void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t
   cudaStream_t s = (cudaStream_t)stream;
   if (comm->mode != 1) {
     if (count == 0) return;
+    if (algo->s->opt.nvls && try_nvls(comm, *algo->s, coll, send, recv, count, dt, op, s)) return;
     launch_rank(comm, algo, CallDesc{coll, count, dt, op}, send, recv, s);
     return;
   }
@@ -853,6 +863,288 @@ Plan plan_from(const char* irText, const char* opts, Options* o_out, Ir* ir_out)
   if (o_out) *o_out = o;
   if (ir_out) *ir_out = ir;
   return p;
+}
+
+
+// ---------------------------------------------------------------- f3: NVLS windows and transport
+// SURVEY §8(f) f3 (not in the paper): the NVSwitch-SHARP variant of the transport.  An
+// NVLS window is device memory of every rank bound into one multicast object; calls of
+// an algorithm loaded with nvls=1 whose buffers lie in NVLS windows run the NVLS kernel
+// (rdev::nvls_run: mred / mcast on the collective's chunk layout), every other call runs
+// the algorithm's primitive plan.  Driver entry points are resolved on first use so a
+// driver without multicast only fails the NVLS calls.
+constexpr size_t kNvlsHdr = 4096;  // barrier words [entry, exit] at the window's start
+
+struct NvlsDriver {
+  CUresult (*McCreate)(CUmemGenericAllocationHandle*, const CUmulticastObjectProp*) = nullptr;
+  CUresult (*McAddDevice)(CUmemGenericAllocationHandle, CUdevice) = nullptr;
+  CUresult (*McBindMem)(CUmemGenericAllocationHandle, size_t, CUmemGenericAllocationHandle, size_t, size_t,
+                        unsigned long long) = nullptr;
+  CUresult (*McUnbind)(CUmemGenericAllocationHandle, CUdevice, size_t, size_t) = nullptr;
+  CUresult (*McGetGranularity)(size_t*, const CUmulticastObjectProp*, CUmulticastGranularity_flags) = nullptr;
+  CUresult (*MemCreate)(CUmemGenericAllocationHandle*, size_t, const CUmemAllocationProp*, unsigned long long) =
+      nullptr;
+  CUresult (*MemRelease)(CUmemGenericAllocationHandle) = nullptr;
+  CUresult (*MemAddressReserve)(CUdeviceptr*, size_t, size_t, CUdeviceptr, unsigned long long) = nullptr;
+  CUresult (*MemAddressFree)(CUdeviceptr, size_t) = nullptr;
+  CUresult (*MemMap)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle, unsigned long long) = nullptr;
+  CUresult (*MemUnmap)(CUdeviceptr, size_t) = nullptr;
+  CUresult (*MemSetAccess)(CUdeviceptr, size_t, const CUmemAccessDesc*, size_t) = nullptr;
+  CUresult (*MemExport)(void*, CUmemGenericAllocationHandle, CUmemAllocationHandleType, unsigned long long) =
+      nullptr;
+  CUresult (*MemImport)(CUmemGenericAllocationHandle*, void*, CUmemAllocationHandleType) = nullptr;
+  CUresult (*DeviceGet)(CUdevice*, int) = nullptr;
+  CUresult (*DeviceGetAttribute)(int*, CUdevice_attribute, CUdevice) = nullptr;
+};
+
+NvlsDriver& nvls_driver() {
+  static NvlsDriver d;
+  static bool ok = false;
+  if (!ok) {
+    driver();  // the base entry points first (fails cleanly without a driver)
+    entry("cuMulticastCreate", &d.McCreate);
+    entry("cuMulticastAddDevice", &d.McAddDevice);
+    entry("cuMulticastBindMem", &d.McBindMem);
+    entry("cuMulticastUnbind", &d.McUnbind);
+    entry("cuMulticastGetGranularity", &d.McGetGranularity);
+    entry("cuMemCreate", &d.MemCreate);
+    entry("cuMemRelease", &d.MemRelease);
+    entry("cuMemAddressReserve", &d.MemAddressReserve);
+    entry("cuMemAddressFree", &d.MemAddressFree);
+    entry("cuMemMap", &d.MemMap);
+    entry("cuMemUnmap", &d.MemUnmap);
+    entry("cuMemSetAccess", &d.MemSetAccess);
+    entry("cuMemExportToShareableHandle", &d.MemExport);
+    entry("cuMemImportFromShareableHandle", &d.MemImport);
+    entry("cuDeviceGet", &d.DeviceGet);
+    entry("cuDeviceGetAttribute", &d.DeviceGetAttribute);
+    ok = true;
+  }
+  return d;
+}
+
+// one multicast object; released when the last window bound to it is released
+struct McObj {
+  CUmemGenericAllocationHandle h = 0;
+  ~McObj() {
+    if (h) nvls_driver().MemRelease(h);
+  }
+};
+
+struct NvlsWin {
+  std::shared_ptr<McObj> mc_obj;
+  int dev = 0;
+  size_t bytes = 0, total = 0;  // user bytes; mapped bytes (header + user, granularity-rounded)
+  CUmemGenericAllocationHandle mc = 0, mem = 0;
+  CUdeviceptr uc = 0, mcva = 0;
+  bool added = false, bound = false, uc_mapped = false, mc_mapped = false;
+  unsigned arrivals = 0;  // barrier arrivals per word after the calls issued so far
+  char* user() const { return (char*)uc + kNvlsHdr; }
+  char* user_mc() const { return (char*)mcva + kNvlsHdr; }
+};
+
+CUmulticastObjectProp nvls_prop(int nranks, size_t total, bool fabric) {
+  CUmulticastObjectProp p;
+  memset(&p, 0, sizeof(p));
+  p.numDevices = (unsigned)nranks;
+  p.size = total;
+  p.handleTypes = fabric ? CU_MEM_HANDLE_TYPE_FABRIC : CU_MEM_HANDLE_TYPE_NONE;
+  return p;
+}
+
+size_t nvls_total(int nranks, size_t bytes, bool fabric) {
+  CUmulticastObjectProp p = nvls_prop(nranks, kNvlsHdr + bytes, fabric);
+  size_t g = 0;
+  cu_check(nvls_driver().McGetGranularity(&g, &p, CU_MULTICAST_GRANULARITY_RECOMMENDED),
+           "cuMulticastGetGranularity");
+  if (g == 0) g = 2 << 20;
+  return (kNvlsHdr + bytes + g - 1) / g * g;
+}
+
+void nvls_add_device(NvlsWin& w) {
+  CUdevice d;
+  cu_check(nvls_driver().DeviceGet(&d, w.dev), "cuDeviceGet");
+  cu_check(nvls_driver().McAddDevice(w.mc, d), "cuMulticastAddDevice");
+  w.added = true;
+}
+
+// after every rank's device is added: this rank's memory, bound and mapped twice
+void nvls_bind_map(NvlsWin& w) {
+  NvlsDriver& D = nvls_driver();
+  cuda_check(cudaSetDevice(w.dev), "cudaSetDevice");
+  CUmemAllocationProp ap;
+  memset(&ap, 0, sizeof(ap));
+  ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  ap.location.id = w.dev;
+  cu_check(D.MemCreate(&w.mem, w.total, &ap, 0), "cuMemCreate");
+  cu_check(D.McBindMem(w.mc, 0, w.mem, 0, w.total, 0), "cuMulticastBindMem");
+  w.bound = true;
+  CUmemAccessDesc ad;
+  memset(&ad, 0, sizeof(ad));
+  ad.location = ap.location;
+  ad.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  cu_check(D.MemAddressReserve(&w.uc, w.total, 2 << 20, 0, 0), "cuMemAddressReserve");
+  cu_check(D.MemMap(w.uc, w.total, 0, w.mem, 0), "cuMemMap(unicast)");
+  w.uc_mapped = true;
+  cu_check(D.MemSetAccess(w.uc, w.total, &ad, 1), "cuMemSetAccess(unicast)");
+  cu_check(D.MemAddressReserve(&w.mcva, w.total, 2 << 20, 0, 0), "cuMemAddressReserve");
+  cu_check(D.MemMap(w.mcva, w.total, 0, w.mc, 0), "cuMemMap(multicast)");
+  w.mc_mapped = true;
+  cu_check(D.MemSetAccess(w.mcva, w.total, &ad, 1), "cuMemSetAccess(multicast)");
+  cuda_check(cudaMemset((void*)w.uc, 0, kNvlsHdr), "cudaMemset(nvls header)");
+  cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
+}
+
+// best effort: every step that was taken is undone
+void nvls_release(NvlsWin& w) {
+  NvlsDriver& D = nvls_driver();
+  cudaSetDevice(w.dev);
+  cudaDeviceSynchronize();
+  if (w.mc_mapped) D.MemUnmap(w.mcva, w.total);
+  if (w.mcva) D.MemAddressFree(w.mcva, w.total);
+  if (w.uc_mapped) D.MemUnmap(w.uc, w.total);
+  if (w.uc) D.MemAddressFree(w.uc, w.total);
+  if (w.bound) {
+    CUdevice d;
+    if (D.DeviceGet(&d, w.dev) == CUDA_SUCCESS) D.McUnbind(w.mc, d, 0, w.total);
+  }
+  if (w.mem) D.MemRelease(w.mem);
+  w = NvlsWin();  // drops this window's reference to the multicast object
+}
+
+// the NVLS window of `comm` holding [p, p + bytes), or null
+NvlsWin* nvls_find(rescclComm* comm, const void* p, size_t bytes) {
+  for (auto& w : comm->nvls)
+    if ((const char*)p >= w->user() && (const char*)p + bytes <= w->user() + w->bytes) return w.get();
+  return nullptr;
+}
+
+std::string nvls_source(int coll) {
+  return "#include \"resccl_device.cuh\"\n"
+         "extern \"C\" __global__ void __launch_bounds__(512, 1) resccl_nvls_kernel(rdev::NvlsArgs a) {\n"
+         "  rdev::nvls_run<RESCCL_T, RESCCL_OP, " +
+         std::to_string(coll) + ">(a);\n}\n";
+}
+
+Kern& nvls_kernel(int dev, int coll, rescclDataType_t dt, rescclRedOp_t op) {
+  static std::map<std::string, Kern> cache;  // per device (modules are per context)
+  std::string key = std::to_string(dev) + "/" + std::to_string(coll) + "/" + std::to_string((int)dt) + "/" +
+                    std::to_string((int)op);
+  auto it = cache.find(key);
+  if (it != cache.end()) return it->second;
+  std::vector<char> cubin = nvrtc_compile(nvls_source(coll), dt, op, false);
+  Kern k;
+  cu_check(driver().ModuleLoadData(&k.mod, cubin.data()), "cuModuleLoadData(nvls)");
+  cu_check(driver().ModuleGetFunction(&k.fn, k.mod, "resccl_nvls_kernel"), "cuModuleGetFunction(nvls)");
+  return cache[key] = k;
+}
+
+struct NvlsArgsHost {  // mirrors rdev::NvlsArgs
+  char* mc_send;
+  char* mc_recv;
+  const char* uc_send;
+  char* uc_recv;
+  unsigned* mc_flags;
+  unsigned* uc_flags;
+  long long lo_bytes, hi_bytes;
+  unsigned target;
+  int nranks;
+  int vec;
+  int* err;
+  unsigned long long timeout_ns;
+};
+
+// NVLS eligibility of a call (rank-independent, so every rank decides alike) and launch.
+// Returns false -- the caller runs the primitive plan -- when a buffer is outside the NVLS
+// windows or at an offset that is not 4-byte aligned, a per-rank block is not whole
+// 4-byte granules, or the op has no multimem form (f32 max/min).
+bool try_nvls(rescclComm* comm, const AlgoShared& a, int coll, const void* send, void* recv, size_t count,
+              rescclDataType_t dt, rescclRedOp_t op, cudaStream_t s) {
+  if (comm->nvls.empty() || comm->mode == 1) return false;
+  if (dt == rescclFloat32 && op != rescclSum) return false;
+  const int N = comm->nranks, r = comm->rank;
+  const long long e = elt_size(dt);
+  const long long blk = (long long)count * e;  // AR: whole buffer; RS/AG: one rank's block
+  const long long sbytes = coll == (int)Coll::ReduceScatter ? blk * N : blk;
+  const long long rbytes = coll == (int)Coll::AllGather ? blk * N : blk;
+  if (blk % 4) return false;
+  // every buffer in an NVLS window (also RS's receive and AG's send buffer, which are
+  // only touched locally): windows are symmetric, so the decision below is the same on
+  // every rank
+  NvlsWin* ws = nvls_find(comm, send, (size_t)sbytes);
+  NvlsWin* wr = nvls_find(comm, recv, (size_t)rbytes);
+  if (!ws || !wr) return false;
+  const long long os = (const char*)send - ws->user();
+  const long long orr = (char*)recv - wr->user();
+  if (os % 4 || orr % 4) return false;
+  NvlsWin& W = coll == (int)Coll::ReduceScatter ? *ws : *wr;  // carries the barrier words
+  NvlsArgsHost ka;
+  memset(&ka, 0, sizeof(ka));
+  ka.mc_send = ws->user_mc() + os;
+  ka.mc_recv = wr->user_mc() + orr;
+  ka.uc_send = (const char*)send;
+  ka.uc_recv = (char*)recv;
+  ka.mc_flags = (unsigned*)W.mcva;
+  ka.uc_flags = (unsigned*)W.uc;
+  long long span;  // largest per-rank range (rank-independent grid)
+  if (coll == (int)Coll::AllReduce) {
+    // AR partition: 16-byte-aligned slices of ceil(S/N) (reading R28); any partition gives
+    // the same result, each element is reduced by exactly one rank
+    const long long sl = ((blk + N - 1) / N + 15) / 16 * 16;
+    ka.lo_bytes = std::min(r * sl, blk);
+    ka.hi_bytes = std::min(ka.lo_bytes + sl, blk);
+    ka.vec = os % 16 == 0 && orr % 16 == 0;
+    span = sl;
+  } else {
+    ka.lo_bytes = r * blk;
+    ka.hi_bytes = ka.lo_bytes + blk;
+    ka.vec = blk % 16 == 0 && os % 16 == 0 && orr % 16 == 0;
+    span = blk;
+  }
+  const long long per_cta = 512LL * 4 * (ka.vec ? 16 : 4);
+  const int grid = (int)std::max(1LL, std::min((long long)a.opt.nvls_ctas, (span + per_cta - 1) / per_cta));
+  W.arrivals += (unsigned)(N * grid);
+  ka.target = W.arrivals;
+  ka.nranks = N;
+  ka.err = comm->err_dev;
+  ka.timeout_ns = timeout_ns();
+  cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+  Kern& k = nvls_kernel(comm->dev, coll, dt, op);
+  void* params[] = {&ka};
+  cu_check(driver().LaunchCooperativeKernel(k.fn, grid, 1, 1, 512, 1, 1, 0, (CUstream)s, params),
+           "cuLaunchCooperativeKernel(nvls)");
+  return true;
+}
+
+// Multi-process NVLS window: rank 0 creates the multicast object and exports a fabric
+// handle; every rank imports it, adds its device, then binds and maps its memory.  Every
+// rank runs all three exchanges whatever happened locally, so a failure on any rank
+// surfaces on every rank (same order of callback calls, no hang).
+struct NvlsBlob {
+  unsigned magic;
+  int ok;
+  unsigned long long total;
+  CUmemFabricHandle handle;
+  char msg[160];
+};
+
+void nvls_status(NvlsBlob& b, const std::string& m) {
+  b.ok = 0;
+  snprintf(b.msg, sizeof(b.msg), "%s", m.c_str());
+}
+
+void nvls_exchange(NvlsBlob& mine, std::vector<NvlsBlob>& all, int nranks,
+                   int (*allgather)(const void*, void*, size_t, void*), void* ctx, const char* phase) {
+  all.assign(nranks, NvlsBlob());
+  if (allgather(&mine, all.data(), sizeof(NvlsBlob), ctx) != 0)
+    fail(rescclSystemError, std::string("allgather callback failed (") + phase + ")");
+  for (int q = 0; q < nranks; ++q) {
+    if (all[q].magic != 0x4e564c53u) fail(rescclSystemError, std::string("corrupt NVLS blob (") + phase + ")");
+    if (!all[q].ok)
+      fail(rescclCudaError, std::string("NVLS window (") + phase + ") failed on rank " + std::to_string(q) + ": " +
+                                std::string(all[q].msg, strnlen(all[q].msg, sizeof(all[q].msg))));
+  }
 }
 
 }  // namespace
@@ -1130,6 +1422,8 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
   if (!comm) return rescclSuccess;
   cudaSetDevice(comm->dev);
   cudaDeviceSynchronize();
+  for (auto& w : comm->nvls) nvls_release(*w);
+  comm->nvls.clear();
   if (comm->mode == 1) {
     Group* G = comm->group;
     if (--G->refs == 0) {
@@ -1273,6 +1567,146 @@ rescclResult_t rescclReduceScatter(const void* sendbuf, void* recvbuf, size_t re
 }
 
 // ------------------------------------------------------------------ host-only tools
+// ---------------------------------------------------------------- f3: NVLS windows
+rescclResult_t rescclNvlsSupported(rescclComm_t comm, int* supported) {
+  API_BEGIN
+  if (!comm || !supported) fail(rescclInvalidArgument, "null argument");
+  *supported = 0;
+  if (comm->mode == 1) return rescclSuccess;  // virtual ranks share one device
+  NvlsDriver& D = nvls_driver();
+  CUdevice d;
+  cu_check(D.DeviceGet(&d, comm->dev), "cuDeviceGet");
+  int v = 0;
+  cu_check(D.DeviceGetAttribute(&v, CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED, d), "cuDeviceGetAttribute");
+  *supported = v;
+  API_END
+}
+
+rescclResult_t rescclNvlsAlloc(rescclComm_t comm, size_t bytes, int (*allgather)(const void*, void*, size_t, void*),
+                               void* ctx, void** ptr) {
+  API_BEGIN
+  if (!comm || !allgather || !ptr) fail(rescclInvalidArgument, "null argument");
+  if (bytes == 0) fail(rescclInvalidArgument, "empty NVLS window");
+  if (comm->mode != 0) fail(rescclInvalidUsage, "rescclNvlsAlloc is for multi-process communicators (see rescclNvlsAllocAll)");
+  *ptr = nullptr;
+  auto w = std::make_shared<NvlsWin>();
+  w->dev = comm->dev;
+  w->bytes = bytes;
+  NvlsBlob mine;
+  memset(&mine, 0, sizeof(mine));
+  mine.magic = 0x4e564c53u;
+  mine.ok = 1;
+  std::vector<NvlsBlob> all;
+  try {
+    // 1: rank 0 creates and exports the multicast object; everyone agrees on its size
+    try {
+      cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+      w->total = nvls_total(comm->nranks, bytes, true);
+      mine.total = w->total;
+      if (comm->rank == 0) {
+        CUmulticastObjectProp p = nvls_prop(comm->nranks, w->total, true);
+        cu_check(nvls_driver().McCreate(&w->mc, &p), "cuMulticastCreate");
+        w->mc_obj = std::make_shared<McObj>();
+        w->mc_obj->h = w->mc;
+        cu_check(nvls_driver().MemExport(&mine.handle, w->mc, CU_MEM_HANDLE_TYPE_FABRIC, 0),
+                 "cuMemExportToShareableHandle(fabric)");
+      }
+    } catch (Error& e) {
+      nvls_status(mine, e.msg);
+    }
+    nvls_exchange(mine, all, comm->nranks, allgather, ctx, "create");
+    for (auto& b : all)
+      if (b.total != w->total) fail(rescclInvalidUsage, "NVLS windows must have the same size on every rank");
+    // 2: import and add this rank's device
+    try {
+      if (comm->rank != 0) {
+        cu_check(nvls_driver().MemImport(&w->mc, &all[0].handle, CU_MEM_HANDLE_TYPE_FABRIC),
+                 "cuMemImportFromShareableHandle(fabric)");
+        w->mc_obj = std::make_shared<McObj>();
+        w->mc_obj->h = w->mc;
+      }
+      nvls_add_device(*w);
+    } catch (Error& e) {
+      nvls_status(mine, e.msg);
+    }
+    nvls_exchange(mine, all, comm->nranks, allgather, ctx, "add device");
+    // 3: bind and map (every device is in the object now)
+    try {
+      nvls_bind_map(*w);
+    } catch (Error& e) {
+      nvls_status(mine, e.msg);
+    }
+    nvls_exchange(mine, all, comm->nranks, allgather, ctx, "bind");
+  } catch (...) {
+    nvls_release(*w);
+    throw;
+  }
+  comm->nvls.push_back(w);
+  *ptr = w->user();
+  API_END
+}
+
+rescclResult_t rescclNvlsAllocAll(rescclComm_t* comms, int n, size_t bytes, void** ptrs) {
+  API_BEGIN
+  if (!comms || !ptrs || n < 1) fail(rescclInvalidArgument, "bad arguments");
+  if (bytes == 0) fail(rescclInvalidArgument, "empty NVLS window");
+  for (int k = 0; k < n; ++k) {
+    if (!comms[k] || comms[k]->rank != k || comms[k]->nranks != n)
+      fail(rescclInvalidArgument, "comms must be ranks 0..n-1 of one communicator");
+    if (comms[k]->mode != 2) fail(rescclInvalidUsage, "rescclNvlsAllocAll needs one device per rank (rescclCommInitAll with distinct devices)");
+  }
+  std::vector<std::shared_ptr<NvlsWin>> ws(n);
+  try {
+    cuda_check(cudaSetDevice(comms[0]->dev), "cudaSetDevice");
+    const size_t total = nvls_total(n, bytes, false);
+    CUmulticastObjectProp p = nvls_prop(n, total, false);
+    auto mco = std::make_shared<McObj>();
+    cu_check(nvls_driver().McCreate(&mco->h, &p), "cuMulticastCreate");
+    const CUmemGenericAllocationHandle mc = mco->h;
+    for (int k = 0; k < n; ++k) {
+      ws[k] = std::make_shared<NvlsWin>();
+      ws[k]->mc_obj = mco;
+      ws[k]->dev = comms[k]->dev;
+      ws[k]->bytes = bytes;
+      ws[k]->total = total;
+      ws[k]->mc = mc;
+    }
+    for (int k = 0; k < n; ++k) nvls_add_device(*ws[k]);
+    for (int k = 0; k < n; ++k) nvls_bind_map(*ws[k]);
+  } catch (...) {
+    for (int k = n - 1; k >= 0; --k)
+      if (ws[k]) nvls_release(*ws[k]);
+    throw;
+  }
+  for (int k = 0; k < n; ++k) {
+    comms[k]->nvls.push_back(ws[k]);
+    ptrs[k] = ws[k]->user();
+  }
+  API_END
+}
+
+rescclResult_t rescclNvlsFree(rescclComm_t comm, void* ptr) {
+  API_BEGIN
+  if (!comm || !ptr) fail(rescclInvalidArgument, "null argument");
+  for (size_t i = 0; i < comm->nvls.size(); ++i)
+    if (comm->nvls[i]->user() == (char*)ptr) {
+      nvls_release(*comm->nvls[i]);
+      comm->nvls.erase(comm->nvls.begin() + i);
+      return rescclSuccess;
+    }
+  fail(rescclInvalidArgument, "not an NVLS window of this communicator");
+  API_END
+}
+
+rescclResult_t rescclCompileNvls(rescclColl_t coll, rescclDataType_t dtype, rescclRedOp_t op, size_t* cubin_bytes) {
+  API_BEGIN
+  if (!cubin_bytes) fail(rescclInvalidArgument, "null argument");
+  if ((int)coll < 0 || (int)coll > 2 || elt_size(dtype) == 0 || (int)op < 0 || (int)op > 2)
+    fail(rescclInvalidArgument, "bad coll/dtype/op");
+  *cubin_bytes = nvrtc_compile(nvls_source((int)coll), dtype, op, false).size();
+  API_END
+}
+
 rescclResult_t rescclGenerateIr(const char* name, rescclColl_t coll, int nranks, const char* opts, char* text,
                                 size_t* len) {
   API_BEGIN

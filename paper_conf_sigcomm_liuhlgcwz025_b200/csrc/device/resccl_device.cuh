@@ -1330,4 +1330,181 @@ __device__ __noinline__ void exit_barrier(const KArgs& a, int rank, int nranks, 
   }
 }
 
+// ============================================================================= f3: NVLS transport
+// NVLink SHARP (not in the paper, the B200 NVSwitch variant of the
+// transport).  Every rank's buffer is bound into one multicast object, so a load through
+// the multicast alias (multimem.ld_reduce) returns the reduction of all ranks' copies,
+// computed inside the switch, and a store through it (multimem.st) lands in every rank's
+// copy.  On the collective's chunk layout (R6: chunk c belongs to rank c) the schedule is
+//   mred(r): <r,c=r> := (+)_k <k,r>     (ReduceScatter; one multimem.ld_reduce per granule)
+//   mcast(r): <k,r>  := <r,r>  for all k (AllGather; one multimem.st per granule)
+// and AllReduce = mred then mcast of each rank's own chunk.  mcast(r)
+// depends only on mred(r) of the same granule in the same thread, so no barrier sits
+// between the phases; an entry barrier orders every rank's earlier writes of its send
+// buffer before anyone's multimem loads, and an exit barrier keeps a rank's kernel alive
+// until every peer's multicast stores into its receive buffer have landed.
+// Granules are 16 bytes (v4) when every address is 16-byte aligned, else 4 bytes; the
+// host only routes calls whose per-rank blocks are whole 4-byte granules here (2-byte
+// dtypes: even counts) and f32 max/min, which multimem.ld_reduce lacks, elsewhere.
+struct NvlsArgs {
+  char* mc_send;         // multicast alias of sendbuf (AR/RS) -- null for AG
+  char* mc_recv;         // multicast alias of recvbuf (AR/AG) -- null for RS
+  const char* uc_send;   // this rank's sendbuf (AG source)
+  char* uc_recv;         // this rank's recvbuf (RS destination)
+  u32* mc_flags;         // multicast alias of the window's barrier words [entry, exit]
+  u32* uc_flags;         // this rank's copy of them
+  i64 lo_bytes;          // this rank's byte range [lo, hi) of the AR buffer / RS,AG block
+  i64 hi_bytes;
+  u32 target;            // barrier arrivals on this window once this call's have landed
+  int nranks;
+  int vec;               // 1: 16-byte granules, 0: 4-byte granules
+  int* err;
+  u64 timeout_ns;
+};
+
+template <class T, int OP>
+__device__ __forceinline__ void mm_ldred4(const char* mc, u32 (&v)[4]);
+template <class T, int OP>
+__device__ __forceinline__ u32 mm_ldred1(const char* mc);
+
+#define RESCCL_MM_V4(SUF)                                                                   \
+  asm volatile("multimem.ld_reduce.relaxed.sys.global." SUF " {%0,%1,%2,%3}, [%4];"          \
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "l"(mc) : "memory")
+#define RESCCL_MM_S4(SUF)                                                                   \
+  asm volatile("multimem.ld_reduce.relaxed.sys.global." SUF " %0, [%1];" : "=r"(x) : "l"(mc) : "memory")
+#define RESCCL_MM_INT4(SUF)                                                                 \
+  for (int j = 0; j < 4; ++j)                                                               \
+    asm volatile("multimem.ld_reduce.relaxed.sys.global." SUF " %0, [%1];"                  \
+                 : "=r"(v[j]) : "l"(mc + 4 * j) : "memory")
+
+// bf16 / f16 sums accumulate in fp32 inside the switch and round once (acc::f32)
+template <> __device__ __forceinline__ void mm_ldred4<TBF16, OpSum>(const char* mc, u32 (&v)[4]) { RESCCL_MM_V4("add.acc::f32.v4.bf16x2"); }
+template <> __device__ __forceinline__ void mm_ldred4<TBF16, OpMax>(const char* mc, u32 (&v)[4]) { RESCCL_MM_V4("max.v4.bf16x2"); }
+template <> __device__ __forceinline__ void mm_ldred4<TBF16, OpMin>(const char* mc, u32 (&v)[4]) { RESCCL_MM_V4("min.v4.bf16x2"); }
+template <> __device__ __forceinline__ void mm_ldred4<TF16, OpSum>(const char* mc, u32 (&v)[4]) { RESCCL_MM_V4("add.acc::f32.v4.f16x2"); }
+template <> __device__ __forceinline__ void mm_ldred4<TF16, OpMax>(const char* mc, u32 (&v)[4]) { RESCCL_MM_V4("max.v4.f16x2"); }
+template <> __device__ __forceinline__ void mm_ldred4<TF16, OpMin>(const char* mc, u32 (&v)[4]) { RESCCL_MM_V4("min.v4.f16x2"); }
+template <> __device__ __forceinline__ void mm_ldred4<TF32, OpSum>(const char* mc, u32 (&v)[4]) { RESCCL_MM_V4("add.v4.f32"); }
+template <> __device__ __forceinline__ void mm_ldred4<TI32, OpSum>(const char* mc, u32 (&v)[4]) { RESCCL_MM_INT4("add.u32"); }
+template <> __device__ __forceinline__ void mm_ldred4<TI32, OpMax>(const char* mc, u32 (&v)[4]) { RESCCL_MM_INT4("max.s32"); }
+template <> __device__ __forceinline__ void mm_ldred4<TI32, OpMin>(const char* mc, u32 (&v)[4]) { RESCCL_MM_INT4("min.s32"); }
+template <> __device__ __forceinline__ u32 mm_ldred1<TBF16, OpSum>(const char* mc) { u32 x; RESCCL_MM_S4("add.acc::f32.bf16x2"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TBF16, OpMax>(const char* mc) { u32 x; RESCCL_MM_S4("max.bf16x2"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TBF16, OpMin>(const char* mc) { u32 x; RESCCL_MM_S4("min.bf16x2"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TF16, OpSum>(const char* mc) { u32 x; RESCCL_MM_S4("add.acc::f32.f16x2"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TF16, OpMax>(const char* mc) { u32 x; RESCCL_MM_S4("max.f16x2"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TF16, OpMin>(const char* mc) { u32 x; RESCCL_MM_S4("min.f16x2"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TF32, OpSum>(const char* mc) { u32 x; RESCCL_MM_S4("add.f32"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TI32, OpSum>(const char* mc) { u32 x; RESCCL_MM_S4("add.u32"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TI32, OpMax>(const char* mc) { u32 x; RESCCL_MM_S4("max.s32"); return x; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TI32, OpMin>(const char* mc) { u32 x; RESCCL_MM_S4("min.s32"); return x; }
+// f32 max/min: multimem.ld_reduce has no such form; the host never routes them here
+template <> __device__ __forceinline__ void mm_ldred4<TF32, OpMax>(const char*, u32 (&v)[4]) { v[0] = v[1] = v[2] = v[3] = 0; __trap(); }
+template <> __device__ __forceinline__ void mm_ldred4<TF32, OpMin>(const char*, u32 (&v)[4]) { v[0] = v[1] = v[2] = v[3] = 0; __trap(); }
+template <> __device__ __forceinline__ u32 mm_ldred1<TF32, OpMax>(const char*) { __trap(); return 0; }
+template <> __device__ __forceinline__ u32 mm_ldred1<TF32, OpMin>(const char*) { __trap(); return 0; }
+#undef RESCCL_MM_V4
+#undef RESCCL_MM_S4
+#undef RESCCL_MM_INT4
+
+__device__ __forceinline__ void mm_st4(char* mc, const u32 (&v)[4]) {
+  asm volatile("multimem.st.relaxed.sys.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(mc), "r"(v[0]), "r"(v[1]),
+               "r"(v[2]), "r"(v[3])
+               : "memory");
+}
+__device__ __forceinline__ void mm_st1(char* mc, u32 v) {
+  asm volatile("multimem.st.relaxed.sys.global.b32 [%0], %1;" ::"l"(mc), "r"(v) : "memory");
+}
+
+// Grid-wide NVLS barrier on barrier word w: every block of every rank adds 1 through the
+// multicast alias (release), then waits until its own copy shows all arrivals up to this
+// call's: a.target = (nranks x grid) summed over the window's calls so far, this one
+// included (the host keeps the sum; u32, compared wrap-safe).
+__device__ __forceinline__ void nvls_barrier(const NvlsArgs& a, int w) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    asm volatile("fence.proxy.alias;" ::: "memory");
+    asm volatile("fence.acq_rel.sys;" ::: "memory");
+    asm volatile("multimem.red.release.sys.global.add.u32 [%0], 1;" ::"l"(a.mc_flags + w) : "memory");
+    const u32 target = a.target;
+    const u64 t0 = globaltimer();
+    u32 spins = 0;
+    for (;;) {
+      u32 x;
+      asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(x) : "l"(a.uc_flags + w) : "memory");
+      if ((int)(x - target) >= 0) break;  // wrap-safe
+      if (++spins > 64) nanosleep_(64);
+      if ((spins & 1023) == 0 && globaltimer() - t0 > a.timeout_ns) {
+        atomicCAS(a.err, 0, kErrTimeout);
+        break;
+      }
+    }
+    asm volatile("fence.proxy.alias;" ::: "memory");
+  }
+  __syncthreads();
+}
+
+// One span of granules of G bytes (16: v4, 4: scalar), grid-strided with U granules in
+// flight per thread.  coll: CollAllReduce (mred + mcast), CollReduceScatter (mred ->
+// local), CollAllGather (local -> mcast).  Offsets are byte offsets into the collective's
+// buffer; AR/RS read mc_send + off, AR/AG write mc_recv + off, RS writes
+// uc_recv + (off - lo), AG reads uc_send + (off - lo).
+template <class T, int OP, int COLL, int G>
+__device__ __forceinline__ void nvls_span(const NvlsArgs& a, i64 from, i64 to) {
+  const i64 tid = (i64)blockIdx.x * blockDim.x + threadIdx.x;
+  const i64 nth = (i64)gridDim.x * blockDim.x;
+  const i64 lo = a.lo_bytes;
+  const i64 n = (to - from) / G;
+  constexpr int U = 4;
+  for (i64 base = tid; base < n; base += nth * U) {
+    u32 v[U][4];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const i64 k = base + (i64)u * nth;
+      if (k < n) {
+        const i64 off = from + k * G;
+        if (COLL == CollAllGather) {
+          if (G == 16) {
+            const uint4 w = *reinterpret_cast<const uint4*>(a.uc_send + (off - lo));
+            v[u][0] = w.x; v[u][1] = w.y; v[u][2] = w.z; v[u][3] = w.w;
+          } else {
+            v[u][0] = *reinterpret_cast<const u32*>(a.uc_send + (off - lo));
+          }
+        } else if (G == 16) {
+          mm_ldred4<T, OP>(a.mc_send + off, v[u]);
+        } else {
+          v[u][0] = mm_ldred1<T, OP>(a.mc_send + off);
+        }
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const i64 k = base + (i64)u * nth;
+      if (k < n) {
+        const i64 off = from + k * G;
+        if (COLL == CollReduceScatter) {
+          if (G == 16) *reinterpret_cast<uint4*>(a.uc_recv + (off - lo)) = make_uint4(v[u][0], v[u][1], v[u][2], v[u][3]);
+          else *reinterpret_cast<u32*>(a.uc_recv + (off - lo)) = v[u][0];
+        } else if (G == 16) {
+          mm_st4(a.mc_recv + off, v[u]);
+        } else {
+          mm_st1(a.mc_recv + off, v[u][0]);
+        }
+      }
+    }
+  }
+}
+
+// This rank's range [lo, hi): 16-byte granules from lo (vec; lo is 16-byte aligned in
+// every address space then) and 4-byte granules for the rest.
+template <class T, int OP, int COLL>
+__device__ __forceinline__ void nvls_run(const NvlsArgs& a) {
+  nvls_barrier(a, 0);
+  const i64 lo = a.lo_bytes, hi = a.hi_bytes;
+  const i64 mid = a.vec ? lo + (hi - lo) / 16 * 16 : lo;
+  if (a.vec) nvls_span<T, OP, COLL, 16>(a, lo, mid);
+  nvls_span<T, OP, COLL, 4>(a, mid, hi);
+  nvls_barrier(a, 1);
+}
+
 }  // namespace rdev

@@ -68,6 +68,17 @@ class Communicator:
         dist.all_gather_object(blobs, blob, group=group)
         return _r.rescclCommRegisterConnect(self.handle, blobs)
 
+    def nvls_alloc(self, nbytes: int, group=None) -> int:
+        """Allocate an NVLS window (f3; collective over the process group): the fabric
+        handle and status rounds travel through all_gather_object."""
+        import torch.distributed as dist
+
+        def ag(blob: bytes):
+            out: List[Optional[bytes]] = [None] * self.nranks
+            dist.all_gather_object(out, blob, group=group)
+            return out
+        return _r.rescclNvlsAlloc(self.handle, nbytes, ag)
+
     def destroy(self):
         if self.handle:
             _r.rescclCommDestroy(self.handle)
@@ -106,6 +117,24 @@ class VirtualGroup:
     def destroy(self):
         for c in self.comms:
             c.destroy()
+
+
+class _CudaArray:
+    """__cuda_array_interface__ over a raw device pointer (an NVLS window)."""
+
+    def __init__(self, ptr: int, shape, typestr: str):
+        self.__cuda_array_interface__ = {"data": (ptr, False), "shape": tuple(shape), "typestr": typestr,
+                                         "version": 3, "strides": None}
+
+
+def tensor_at(ptr: int, numel: int, dtype, device: int = 0):
+    """A torch tensor viewing `numel` elements at device pointer `ptr` (not owning it):
+    how NVLS windows are handed to torch.  bf16 has no typestr, so it is viewed via int16."""
+    import torch
+    ts = {torch.float32: "<f4", torch.float16: "<f2", torch.int32: "<i4", torch.bfloat16: "<i2"}[dtype]
+    with torch.cuda.device(device):
+        t = torch.as_tensor(_CudaArray(ptr, (numel,), ts), device=f"cuda:{device}")
+    return t.view(torch.bfloat16) if dtype == torch.bfloat16 else t
 
 
 def init_process_group_comm(rank: int, nranks: int, device: int, group=None) -> Communicator:

@@ -51,10 +51,33 @@ int main(int argc, char** argv) {
   cuDeviceGetAttribute(&fab, CU_DEVICE_ATTRIBUTE_HANDLE_TYPE_FABRIC_SUPPORTED, dev);
   printf("{\"multicast_supported\": %d, \"fabric_handles\": %d}\n", sup, fab);
   size_t sz = 2 << 20;
+  {  // which (handle type, numDevices, size) combinations does cuMulticastCreate accept?
+    const CUmemAllocationHandleType ht[3] = {CU_MEM_HANDLE_TYPE_NONE, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR,
+                                             CU_MEM_HANDLE_TYPE_FABRIC};
+    for (int h = 0; h < 3; ++h)
+      for (int nd = 1; nd <= 2; ++nd)
+        for (size_t s2 = 2 << 20; s2 <= (64u << 20); s2 *= 32) {
+          CUmulticastObjectProp q = {};
+          q.numDevices = nd;
+          q.size = s2;
+          q.handleTypes = ht[h];
+          CUmemGenericAllocationHandle m2;
+          CUresult r = cuMulticastCreate(&m2, &q);
+          const char* nm = 0;
+          cuGetErrorName(r, &nm);
+          printf("{\"create_handle\": %d, \"numDevices\": %d, \"size\": %zu, \"result\": \"%s\"}\n", (int)ht[h], nd, s2, nm);
+          if (r == CUDA_SUCCESS) {
+            CUresult r2 = cuMulticastAddDevice(m2, dev);
+            cuGetErrorName(r2, &nm);
+            printf("{\"add_device\": \"%s\"}\n", nm);
+            cuMemRelease(m2);
+          }
+        }
+  }
   CUmulticastObjectProp mp = {};
   mp.numDevices = twice ? 2 : 1;
   mp.size = sz;
-  mp.handleTypes = CU_MEM_HANDLE_TYPE_NONE;
+  mp.handleTypes = CU_MEM_HANDLE_TYPE_FABRIC;
   size_t g = 0;
   CK(cuMulticastGetGranularity(&g, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED));
   printf("{\"granularity\": %zu}\n", g);
