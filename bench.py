@@ -51,6 +51,9 @@ def parse():
     p.add_argument("--nwarps", type=int, default=0)
     p.add_argument("--tma", type=int, default=-1, help="-1 = library default (on)")
     p.add_argument("--direct", type=int, default=-1, help="direct push/pull transport (default 1; N>1 registers a symmetric window)")
+    p.add_argument("--nvls", type=int, default=0,
+                   help="f3: N>1 only -- send/recv in an NVLS window, NVLS kernel (falls back to --direct if "
+                        "the fabric refuses multicast)")
     p.add_argument("--e2e-steps", type=int, default=3)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--sweep", default="", help="comma-separated MiB sizes for an extra busBW sweep")
@@ -233,7 +236,7 @@ def main():
             "fifodepth": args.fifo_depth or 2,
             "nwarps": args.nwarps or (8 if two_per_sm else None), "tma": None if args.tma < 0 else args.tma,
             "tmastages": 2 if two_per_sm else None, "tmatile": 12288 if two_per_sm else None,
-            "direct": direct}
+            "direct": direct, "nvls": 1 if (args.nvls and multi) else None}
     text = ir_text(R, args.algo, n, opts)
 
     if multi:
@@ -255,7 +258,19 @@ def main():
              if tdt.is_floating_point else torch.randint(-2 ** 20, 2 ** 20, (count,), device=dev, dtype=tdt)
              for r in my_ranks}
     recvs = {r: torch.empty_like(sends[r]) for r in my_ranks}
-    if multi and direct:
+    nvls_state = None
+    if multi and args.nvls:
+        from paper_conf_sigcomm_liuhlgcwz025_b200.torch_api import tensor_at
+        pad = 256 // elt
+        try:
+            ptr = comm.nvls_alloc((2 * count + pad) * elt)
+            win = tensor_at(ptr, 2 * count + pad, tdt, dev.index)
+            win[:count].copy_(sends[rank])
+            sends[rank], recvs[rank] = win[:count], win[count + pad:2 * count + pad]
+            nvls_state = "nvls window"
+        except R.ResCCLError as e:
+            nvls_state = f"unavailable ({e}); direct windows used"
+    if multi and direct and not (nvls_state or "").startswith("nvls"):
         # symmetric window: [send | pad | recv] at the same offsets on every rank
         pad = 256 // elt
         win = torch.empty(2 * count + pad, dtype=tdt, device=dev)
@@ -409,6 +424,8 @@ def main():
     # SMs the kernel occupies: its CTAs (one or two per SM, by block size) spread over the SMs
     n_sm = torch.cuda.get_device_properties(dev).multi_processor_count
     sms = min(n_sm, sum(blocks) if not multi else blocks[rank])
+    if (nvls_state or "").startswith("nvls"):
+        sms = min(n_sm, info.get("nvlsctas", 16))  # upper bound: the grid shrinks for small messages
     line = {
         "metric": "allreduce busBW", "value": round(busbw, 2), "unit": "GB/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
@@ -421,7 +438,9 @@ def main():
                          f"{args.algo} allreduce, {n} GPUs (CUDA-IPC NVLink), {S >> 20} MiB per rank"),
             "nranks": n, "bytes_per_rank": S, "algo": args.algo, "instances": info["instances"],
             "chunkbytes": info["chunkbytes"], "fifodepth": info["fifodepth"], "nwarps": info["nwarps"],
-            "linkmodel": info["linkmodel"], "transport": "direct" if info.get("direct") else "staged-fifo",
+            "linkmodel": info["linkmodel"], "transport": ("nvls" if (nvls_state or "").startswith("nvls") else
+                                                   "direct" if info.get("direct") else "staged-fifo"),
+            **({"nvls": nvls_state} if nvls_state else {}),
             "ctas_per_rank": info["ctas"], "blocks_total": sum(blocks),
             "sms_used": sms, "algbw_gbs": round(algbw, 2), "l2": "inputs > L2 on every rank (no flush)",
             "parallelism": "virtual-ranks" if not multi else f"ranks{n}",

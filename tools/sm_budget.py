@@ -18,6 +18,11 @@ N = 8
 S = int(float(sys.argv[1]) * (1 << 20)) if len(sys.argv) > 1 else 256 << 20
 GEOS = sys.argv[2:] or ["two", "one"]
 GEO = {"two": dict(nwarps=8, tmastages=2, tmatile=12288), "one": dict(nwarps=16, tmastages=4, tmatile=12288)}
+for g in GEOS:  # "w<nwarps>s<stages>t<tile>", e.g. w16s8t6144
+    if g.startswith("w") and "s" in g and "t" in g:
+        w, rest = g[1:].split("s")
+        st, t = rest.split("t")
+        GEO[g] = dict(nwarps=int(w), tmastages=int(st), tmatile=int(t))
 EXTRA = os.environ.get("SMB_OPTS", "")
 COLL = os.environ.get("SMB_COLL", "allreduce")
 INST = [int(x) for x in os.environ.get("SMB_INST", "1,2,3,4,6,8,10,12,16,18,24,30,37").split(",")]
@@ -32,7 +37,7 @@ HB = {"allreduce": 5.0, "reducescatter": 3.0, "allgather": 2.0}[COLL]
 BUSF = {"allreduce": 2.0 * (N - 1) / N}.get(COLL, (N - 1) / N)
 for geo in GEOS:
     for inst in INST:
-        if geo == "one" and inst * N > n_sm:
+        if geo != "two" and inst * N > n_sm:
             continue
         if inst * N > 2 * n_sm:
             continue
