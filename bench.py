@@ -218,24 +218,25 @@ def main():
     count = int(args.size_mb * (1 << 20)) // elt
     S = count * elt
     tdt = getattr(torch, args.dtype)
-    # default tuning: fill the SMs at N=1 (8 virtual ranks share one GPU)
-    # default tuning (r01 sweeps, profiles/r01_*): 18 instances x 8 virtual ranks = 144 CTAs
-    # (of 148 SMs), 4 MiB transfer chunks, FIFO depth 2 (FIFOs stay L2-resident)
-    # The direct transport (R23: push recv payloads, pull rrc operands; no FIFO staging) is
-    # the default: at N=1 every virtual rank's buffers share one address space; under
-    # torchrun (N>1) the send and receive buffers sit in a registered symmetric window.
-    # N=1 (r01 tunes, profiles/r01_pool_tune.txt): two 256-thread CTAs per SM on all 148
-    # SMs (37 instances x 8 ranks = 296 CTAs), each with a 4-stage pool of 24 KiB TMA
-    # stages shared by its two lanes, and 32 MiB transfer chunks (one micro-batch per
-    # 32 MiB algorithm chunk).
+    # Defaults (r01 sweeps, profiles/r01_geo_sweep*.jsonl, profiles/r01_sm_budget_v7.jsonl):
+    # the direct transport (R23: push recv payloads, pull rrc operands; no FIFO staging);
+    # at N=1 every virtual rank's buffers share one address space, under torchrun (N>1) the
+    # send and receive buffers sit in a registered symmetric window.  The lane engine's
+    # cost is per TMA tile, so tiles are 24 KiB (2 stages per lane, one CTA per SM):
+    #   N=1: 18 instances x 8 virtual ranks = 144 CTAs of 256 threads, 32 MiB transfer
+    #        chunks (one micro-batch per 32 MiB algorithm chunk);
+    #   N>1: 24 CTAs of 512 threads per rank (the best per-SM geometry: 87-91 GB/s of HBM
+    #        per SM at <= 32 CTAs), 8 MiB chunks.
     direct = 1 if args.direct < 0 else args.direct
-    two_per_sm = direct and not multi and not args.instances and not args.nwarps
-    inst = args.instances or (37 if two_per_sm else 18)
+    tuned = direct and not args.instances and not args.nwarps
+    inst = args.instances or ((18 if not multi else 24) if tuned else 18)
     opts = {"instances": inst,
-            "chunkbytes": args.chunk_bytes or ((32 << 20) if two_per_sm else (8 << 20) if direct else (4 << 20)),
+            "chunkbytes": args.chunk_bytes or ((32 << 20) if (tuned and not multi) else (8 << 20) if direct
+                                               else (4 << 20)),
             "fifodepth": args.fifo_depth or 2,
-            "nwarps": args.nwarps or (8 if two_per_sm else None), "tma": None if args.tma < 0 else args.tma,
-            "tmastages": 2 if two_per_sm else None, "tmatile": 12288 if two_per_sm else None,
+            "nwarps": args.nwarps or ((8 if not multi else 16) if tuned else None),
+            "tma": None if args.tma < 0 else args.tma,
+            "tmastages": 2 if tuned else None, "tmatile": 24576 if tuned else None,
             "direct": direct, "nvls": 1 if (args.nvls and multi) else None}
     text = ir_text(R, args.algo, n, opts)
 

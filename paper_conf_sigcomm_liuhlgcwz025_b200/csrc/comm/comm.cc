@@ -132,8 +132,9 @@ struct Options {
   bool fuse = true;
   int tb_budget = 0;
   int tma = 1;
-  int tma_tile = 12288;   // r01 sweep: 12 KiB x 4 stages (192 KiB smem per CTA) is best
-  int tma_stages = 4;
+  int tma_tile = 24576;   // r01 geometry sweeps: the engine costs per tile, so 24 KiB x 2 stages per lane
+                          // (192 KiB smem per CTA, one CTA per SM) moves 1.4x the bytes per SM of 12 KiB x 4
+  int tma_stages = 2;
   int trace = 0;
   int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
   int direct = 0;    // direct transport (R23): virtual ranks / single-process only
@@ -144,6 +145,7 @@ struct Options {
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
   int pool_cap = 0;  // stages of the CTA pool one lane may hold (0 = all)
   int ring = 0;      // lane-private TMA stage rings (1) vs one pool shared by both lanes (0)
+  int cpoll = 0;     // combine warps: one polling warp + named barrier (1) vs all polling (0)
   int store_lag = 1; // bulk stores a lane lets drain before it blocks to reuse a stage
   int sys_rank = -1; // rescclCompileIr / rescclCodegenIr: one rank's multi-process (.sys) kernel
   int nvls = 0;      // f3: NVLS transport for calls whose buffers lie in NVLS windows
@@ -195,6 +197,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "poolcap") o.pool_cap = (int)to_long(v, k);
   else if (k == "storelag") o.store_lag = (int)to_long(v, k);
   else if (k == "ring") o.ring = (int)to_long(v, k);
+  else if (k == "cpoll") o.cpoll = (int)to_long(v, k);
   else if (k == "nvls") o.nvls = (int)to_long(v, k);
   else if (k == "nvlsctas") o.nvls_ctas = (int)to_long(v, k);
   else if (k == "sched") {
@@ -217,7 +220,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -498,6 +501,7 @@ CodegenOpts codegen_opts(const Options& o) {
   co.pool_cap = o.pool_cap;
   co.store_lag = o.store_lag;
   co.ring = o.ring;
+  co.cpoll = o.cpoll;
   return co;
 }
 

@@ -722,6 +722,11 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
 #ifndef RESCCL_RING
 #define RESCCL_RING 0
 #endif
+// combine warps: 1 = one warp polls the leader's progress word, the rest wait on a named
+// barrier (ids 3 / 4 = the lane's barrier + 2)
+#ifndef RESCCL_CPOLL
+#define RESCCL_CPOLL 0
+#endif
 // stores a lane lets drain before it blocks on the oldest to reuse its stage
 #ifndef RESCCL_STORE_LAG
 #define RESCCL_STORE_LAG 1
@@ -1109,7 +1114,7 @@ __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const Prim
   const KArgs& a = *L.a;
   const i64 TB = RESCCL_TMA_TILE;  // reduce tiles only
   const u32 Lfull = L.full, Lcomp = L.comp, Lstage = L.stage, Lqprog = L.qprog, Lqdesc = L.qdesc, Lring0 = L.ring0;
-  const int Linst = L.inst, nmb = a.n_mb;
+  const int Linst = L.inst, nmb = a.n_mb, Lbar = L.bar;
   const i64 aM = a.M, aMi = a.Mi, plen = p.len;
   volatile int* const abort_flag = L.abort_flag;
   u32 k = L.tseq;
@@ -1133,10 +1138,24 @@ __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const Prim
       // tiles issued), then map it through that epoch: the epoch holding tile k cannot end
       // before this warp combined it, so the announcing epoch is k's
       u64 w;
+#if RESCCL_CPOLL
+      // one polling warp; the others sleep on the combine warps' named barrier instead of
+      // queueing shared-memory loads behind the TMA traffic
+      if (ctid < 32) {
+        while ((int)((u32)lds_u64(Lqprog) - k) <= 0) {
+          if (++spins > 16) nanosleep_(20);
+          if ((spins & 1023) == 0 && *abort_flag) break;
+        }
+      }
+      asm volatile("bar.sync %0, %1;" ::"r"(Lbar + 2), "r"(nct) : "memory");
+      if (*abort_flag) return false;
+      w = lds_u64(Lqprog);
+#else
       while ((int)((u32)(w = lds_u64(Lqprog)) - k) <= 0) {
         if (++spins > 16) nanosleep_(20);
         if ((spins & 1023) == 0 && *abort_flag) return false;
       }
+#endif
       const u32 eb = (u32)(w >> 32);
       if (eb != cbase) {  // a new epoch: its descriptor (validated by its first tile)
         u64 dsc;

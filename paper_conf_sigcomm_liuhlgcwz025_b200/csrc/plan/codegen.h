@@ -49,8 +49,8 @@ struct CodegenOpts {
   bool gpu_scope = false;        // all ranks on one device (virtual ranks): .gpu-scope flags
   int nwarps = 16;
   int tma = 1;                   // bulk-copy (TMA) data path for non-reducing primitives
-  int tma_tile = 12288;          // bytes per staged tile
-  int tma_stages = 4;            // tiles in flight per lane
+  int tma_tile = 24576;          // bytes per staged tile
+  int tma_stages = 2;            // stages per lane (the CTA pool holds 2x)
   int trace = 0;                 // per-lane lifetime / wait timers (TB utilisation, Table 3)
   int l2hint = 1;                // L2 evict_last on FIFO writes, evict_first on streams
   int tma_min = 163840;          // slices below this many bytes use the register path
@@ -59,6 +59,7 @@ struct CodegenOpts {
   int prefetch = 0;              // micro-batches of local operand prefetched into L2 ahead (off: r01)
   int pool_cap = 0;              // stages of the CTA pool one lane may hold (0 = all)
   int ring = 0;                  // lane-private stage rings instead of the shared CTA pool
+  int cpoll = 0;                 // combine warps: 1 = one polling warp + named barrier
   int store_lag = 1;             // bulk stores a lane lets drain before it blocks to reuse a stage
   int exit_barrier = 0;          // direct transport across processes: a rank's kernel ends only
                                  // after every peer's blocks finished touching its buffers

@@ -147,6 +147,7 @@ int main(int argc, char** argv) {
     }
   };
   run();
+  CK(cudaGetLastError());  // e.g. too many registers for the block size: no timing line
   CK(cudaDeviceSynchronize());
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0); cudaEventCreate(&e1);
