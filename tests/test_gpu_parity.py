@@ -250,3 +250,49 @@ def test_direct_flag_rings_regression(name, coll, kw, fifo):
     assert err == 0 and info["direct"] == 1
     exp = oracle_expect(g, xs, "float32", count, chunk_bytes=8192, instances=2, K=fifo)
     _check_bytes(outs, exp, coll, n, count)
+
+
+@pytest.mark.parametrize("coll", ["allreduce", "allgather", "reducescatter"])
+@pytest.mark.parametrize("direct", [0, 1])
+def test_misaligned_bf16_pointers(coll, direct):
+    """SURVEY d2 tails: bf16 buffers at 2-byte offsets (not 16-byte aligned) take the
+    element path of the register mover and the unaligned TMA tails; bytes = the oracle's."""
+    import torch
+    from gpu_helpers import poison, to_numpy, to_torch
+    n, dtype = 8, "bfloat16"
+    g = oir.generate("ring", coll, n)
+    text = _hdr(g, chunkbytes=1 << 20, instances=2, direct=direct, tmamin=4096)
+    for count in (4097, 300001):
+        xs = _inputs(coll, dtype, n, count, seed=6)
+        grp = R.VirtualGroup(n, 0)
+        try:
+            grp.load(text)
+            sends, recvs = [], []
+            for r in range(n):
+                base = torch.empty(xs[r].size + 1, dtype=torch.bfloat16, device="cuda:0")
+                sends.append(base[1:])  # 2-byte offset
+                sends[-1].copy_(to_torch(xs[r], dtype))
+                m = count * n if coll == "allgather" else count
+                out = torch.empty(m + 3, dtype=torch.bfloat16, device="cuda:0")
+                poison(out)
+                recvs.append(out[3:])  # 6-byte offset
+            getattr(grp, coll)(sends, recvs)
+            torch.cuda.synchronize()
+            assert grp.async_error() == 0
+            outs = [to_numpy(t, dtype) for t in recvs]
+        finally:
+            grp.destroy()
+        exp = oracle_expect(g, xs, dtype, count, chunk_bytes=1 << 20, instances=2)
+        _check_bytes(outs, exp, coll, n, count)
+
+
+def test_count_2pow24_plus_3_direct_allreduce():
+    """SURVEY d2 tail count 2^24 + 3 (bf16, 32 MiB per rank, TMA engine + ragged tail) on
+    exactly representable inputs: every association order gives the definition's bits."""
+    n, dtype, count = 8, "bfloat16", (1 << 24) + 3
+    g = oir.generate("ring", "allreduce", n)
+    text = _hdr(g, chunkbytes=8 << 20, instances=6, direct=1)
+    xs = [inp.rank_input(dtype, 7, r, count, mode="exact") for r in range(n)]
+    outs, _, err = run_virtual(R, text, "allreduce", xs, dtype, count)
+    assert err == 0
+    _check_bytes(outs, definition.allreduce(xs, dtype), "allreduce", n, count)
