@@ -19,6 +19,8 @@ Modules
   definition  collective definitions (sum / concat / scatter)
   numerics    dtype rounding rules used by both definition and replay (R8)
   replay      symbolic + value replay under a blocking FIFO simulator, invariants I1-I6
+  timeline    f2: alpha-beta + Eq. 1 contention timeline, Eq. 7 on wall-clock activity
+  nvls        f3: the NVLS (multimem) schedule -- mred / mcast on the chunk layout (R28)
 
 Parity-unpinned items: HPDS tie-breaks beyond ring/HM/DBT
 (pinned only by readings R3/R4), the choice among equal-size TB colourings, and the
