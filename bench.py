@@ -55,6 +55,8 @@ def parse():
                    help="f3: N>1 only -- send/recv in an NVLS window, NVLS kernel (falls back to --direct if "
                         "the fabric refuses multicast)")
     p.add_argument("--e2e-steps", type=int, default=3)
+    p.add_argument("--inplace-steps", type=int, default=10,
+                   help="also time in-place calls (recv = send) -> config.inplace_busbw_gbs")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--sweep", default="", help="comma-separated MiB sizes for an extra busBW sweep")
     return p.parse_args()
@@ -365,6 +367,32 @@ def main():
         e2e = {"value": round(e2e_bus, 3), "unit": "GB/s", "h2d_bytes_per_step": S * len(my_ranks),
                "d2h_bytes_per_step": S * len(my_ranks), "ms_per_step": round(ems, 3)}
 
+    # ---- in-place (recv = send: the DDP / Megatron bucket case), same workload; the
+    # in-place reduce hops take the bulk-reduction path (bulkred, DESIGN 5.4b)
+    inplace_bus = None
+    if args.inplace_steps > 0:
+        def step_inplace():
+            for r in my_ranks:
+                c = comms[0] if multi else comms[r]
+                c.allreduce(sends[r], sends[r], stream=sid)
+        for _ in range(2):
+            step_inplace()
+        torch.cuda.synchronize(dev)
+        barrier()
+        i0 = torch.cuda.Event(enable_timing=True)
+        i1 = torch.cuda.Event(enable_timing=True)
+        i0.record(stream)
+        for _ in range(args.inplace_steps):
+            step_inplace()
+        i1.record(stream)
+        torch.cuda.synchronize(dev)
+        ims = i0.elapsed_time(i1) / args.inplace_steps
+        if multi:
+            t = torch.tensor([ims], dtype=torch.float64)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            ims = float(t.item())
+        inplace_bus = round(S / (ims * 1e-3) / 1e9 * 2 * (n - 1) / n, 2)
+
     # ---- extra size sweep (busBW vs size)
     sweep = {}
     if args.sweep:
@@ -468,7 +496,7 @@ def main():
                                                    "direct" if info.get("direct") else "staged-fifo"),
             **({"nvls": nvls_state} if nvls_state else {}),
             "ctas_per_rank": info["ctas"], "blocks_total": sum(blocks),
-            "sms_used": sms, "algbw_gbs": round(algbw, 2), "l2": "inputs > L2 on every rank (no flush)",
+            "sms_used": sms, "algbw_gbs": round(algbw, 2), "inplace_busbw_gbs": inplace_bus, "l2": "inputs > L2 on every rank (no flush)",
             "parallelism": "virtual-ranks" if not multi else f"ranks{n}",
         },
         "roofline": roof,

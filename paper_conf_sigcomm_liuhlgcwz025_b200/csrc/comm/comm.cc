@@ -145,6 +145,8 @@ struct Options {
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
   int pool_cap = 0;  // stages of the CTA pool one lane may hold (0 = all)
   int ring = 0;      // lane-private TMA stage rings (1) vs one pool shared by both lanes (0)
+  int bulkred = -1;  // in-place reduce primitives: cp.reduce.async.bulk of the incoming tile
+                     // (-1 = auto: on for AllReduce, where it measured +16% per SM; r01_bulkred_inplace)
   int cpoll = 0;     // combine warps: one polling warp + named barrier (1) vs all polling (0)
   int store_lag = 1; // bulk stores a lane lets drain before it blocks to reuse a stage
   int sys_rank = -1; // rescclCompileIr / rescclCodegenIr: one rank's multi-process (.sys) kernel
@@ -198,6 +200,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "storelag") o.store_lag = (int)to_long(v, k);
   else if (k == "ring") o.ring = (int)to_long(v, k);
   else if (k == "cpoll") o.cpoll = (int)to_long(v, k);
+  else if (k == "bulkred") o.bulkred = (int)to_long(v, k);
   else if (k == "nvls") o.nvls = (int)to_long(v, k);
   else if (k == "nvlsctas") o.nvls_ctas = (int)to_long(v, k);
   else if (k == "sched") {
@@ -220,7 +223,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_BULKRED", "bulkred"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -232,6 +235,7 @@ Options make_options(const Ir& ir, const char* extra) {
       4 * o.tma_tile * o.tma_stages > 200 * 1024)
     fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 4*tile*stages <= 200 KiB");
   if (o.nvls_ctas < 1 || o.nvls_ctas > 148) fail(rescclInvalidArgument, "nvlsctas must be 1..148");
+  if (o.bulkred < 0) o.bulkred = ir.coll == Coll::AllReduce ? 1 : 0;
   if (o.store_lag < 1 || o.store_lag > o.tma_stages)
     fail(rescclInvalidArgument, "storelag must be 1..tmastages");
   return o;
@@ -472,7 +476,7 @@ std::string info_json(const AlgoShared& a) {
   o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
     << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"tma\":" << a.opt.tma
     << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"l2hint\":" << a.opt.l2hint << ",\"prefetch\":" << a.opt.prefetch << ",\"sched\":\""
-    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"nvls\":" << a.opt.nvls << ",\"nvlsctas\":" << a.opt.nvls_ctas << ",\"linkmodel\":\""
+    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"bulkred\":" << a.opt.bulkred << ",\"nvls\":" << a.opt.nvls << ",\"nvlsctas\":" << a.opt.nvls_ctas << ",\"linkmodel\":\""
     << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
     << ",\"ctas\":[";
   for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];
@@ -502,6 +506,7 @@ CodegenOpts codegen_opts(const Options& o) {
   co.store_lag = o.store_lag;
   co.ring = o.ring;
   co.cpoll = o.cpoll;
+  co.bulkred = o.bulkred;
   return co;
 }
 

@@ -603,6 +603,45 @@ template <int F> struct Kind {
   static constexpr int mf = (F & kReduce) | (has_b ? kRecv : 0);      // value = A (+) B, B, or A
 };
 
+// RESCCL_BULKRED: an in-place reduce primitive (local location == store target, nothing
+// forwarded) streams only the incoming tile into shared memory and adds it into the local
+// buffer with one bulk reduction (cp.reduce.async.bulk ... .add, done in L2): no local
+// tile in shared memory and no combine warps.  One correctly rounded add of `local` and
+// `incoming` per element -- the same value as R8's combine (bf16/fp16 .noftz, RN).  f32
+// max/min have no bulk form and keep the combine path.
+#ifndef RESCCL_BULKRED
+#define RESCCL_BULKRED 0
+#endif
+template <class T, int OP>
+struct BulkRed { static constexpr bool ok = !(T::kKind == 1 && OP != OpSum); };
+template <class T, int OP>
+__device__ __forceinline__ void tma_reduce(void* dst, u32 src_smem, u32 bytes, u64 pol);
+#define RESCCL_BRED(TT, O, SUF)                                                                          \
+  template <>                                                                                            \
+  __device__ __forceinline__ void tma_reduce<TT, O>(void* dst, u32 src, u32 bytes, u64 pol) {            \
+    asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.L2::cache_hint." SUF " [%0], [%1], %2, %3;" \
+                 ::"l"(dst), "r"(src), "r"(bytes), "l"(pol) : "memory");                                 \
+  }
+RESCCL_BRED(TBF16, OpSum, "add.noftz.bf16")
+RESCCL_BRED(TBF16, OpMax, "max.bf16")
+RESCCL_BRED(TBF16, OpMin, "min.bf16")
+RESCCL_BRED(TF16, OpSum, "add.noftz.f16")
+RESCCL_BRED(TF16, OpMax, "max.f16")
+RESCCL_BRED(TF16, OpMin, "min.f16")
+RESCCL_BRED(TF32, OpSum, "add.f32")
+RESCCL_BRED(TI32, OpSum, "add.u32")
+RESCCL_BRED(TI32, OpMax, "max.s32")
+RESCCL_BRED(TI32, OpMin, "min.s32")
+#undef RESCCL_BRED
+template <> __device__ __forceinline__ void tma_reduce<TF32, OpMax>(void*, u32, u32, u64) { __trap(); }
+template <> __device__ __forceinline__ void tma_reduce<TF32, OpMin>(void*, u32, u32, u64) { __trap(); }
+// does this reduce primitive take the bulk-reduction path? (leader and combine warps agree)
+template <class T, int OP, int F>
+__device__ __forceinline__ bool bulk_reduce_prim(const char* A, const char* D1) {
+  return RESCCL_BULKRED && (F & kReduce) && (F & kStore) && !Kind<F>::send_data && BulkRed<T, OP>::ok &&
+         A != nullptr && A == D1;
+}
+
 __device__ __forceinline__ u64 dep_target(const KArgs& a, const PrimDesc& d, int k, int j) {
   return (u64)d.dep_n[k] * a.mb_base + (u64)d.dep_pos[k] * a.n_mb + j + 1;
 }
@@ -757,14 +796,18 @@ __device__ __forceinline__ void slice_of_m(i64 M, i64 Mi, i64 len, int j, int in
 }
 // Number of TMA tiles of micro-batch j (16-byte-aligned body only).  A stage holds one
 // reduce tile (A and B halves of RESCCL_TMA_TILE bytes) or one copy tile of twice that.
+// (A bulk-reduced primitive stages only the incoming operand: a whole-stage tile, as a copy.)
 template <int F>
-__device__ __forceinline__ i64 tile_bytes() { return (F & kReduce) ? RESCCL_TMA_TILE : 2 * RESCCL_TMA_TILE; }
+__device__ __forceinline__ i64 tile_bytes(bool bred = false) {
+  return ((F & kReduce) && !bred) ? RESCCL_TMA_TILE : 2 * RESCCL_TMA_TILE;
+}
 template <int F>
-__device__ __forceinline__ u32 mb_tiles_m(i64 M, i64 Mi, i64 len, int j, int inst, int esz, i64& lo, i64& nb) {
+__device__ __forceinline__ u32 mb_tiles_m(i64 M, i64 Mi, i64 len, int j, int inst, int esz, i64& lo, i64& nb,
+                                          bool bred = false) {
   i64 hi;
   slice_of_m(M, Mi, len, j, inst, lo, hi);
   nb = ((hi - lo) * esz) & ~(i64)15;
-  return (u32)((nb + tile_bytes<F>() - 1) / tile_bytes<F>());
+  return (u32)((nb + tile_bytes<F>(bred) - 1) / tile_bytes<F>(bred));
 }
 template <int F>
 __device__ __forceinline__ u32 mb_tiles(const KArgs& a, i64 len, int j, int inst, int esz, i64& lo, i64& nb) {
@@ -799,7 +842,8 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   char* const pin = p.in_data;
   char* const pout = p.out_data;
   const u32 P = RESCCL_POOL;  // slots of the per-tile register records (>= stages held)
-  const i64 TB = tile_bytes<F>();
+  const bool bred = bulk_reduce_prim<T, OP, F>(pA, pD1);
+  const i64 TB = tile_bytes<F>(bred);
   const int nmb = a.n_mb;
   const u32 k0 = L.tseq;
   const u32 sbase = L.stage;
@@ -829,7 +873,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   u32 st = 0;
   int pj = 0;                 // next micro-batch to post
   i64 lo_l = 0, nb_l = 0, lo_s = 0, nb_s = 0, lo_p = 0, nb_p = 0;
-  u32 T_l = mb_tiles_m<F>(aM, aMi, plen, 0, Linst, T::kSize, lo_l, nb_l);
+  u32 T_l = mb_tiles_m<F>(aM, aMi, plen, 0, Linst, T::kSize, lo_l, nb_l, bred);
   u32 T_s = T_l;
   lo_s = lo_l;
   nb_s = nb_l;
@@ -878,7 +922,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       if (lt >= T_l) {
         ++lj;
         lt = 0;
-        if (lj < nmb) T_l = mb_tiles_m<F>(aM, aMi, plen, lj, Linst, T::kSize, lo_l, nb_l);
+        if (lj < nmb) T_l = mb_tiles_m<F>(aM, aMi, plen, lj, Linst, T::kSize, lo_l, nb_l, bred);
         continue;
       }
 #if !RESCCL_RING
@@ -935,7 +979,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
 #if RESCCL_RING
       const u32 s = Lring0 + k % RESCCL_TMA_STAGES;
       const u32 fpar = (k / RESCCL_TMA_STAGES) & 1;
-      if (F & kReduce) {
+      if ((F & kReduce) && !bred) {
         const u32 rb = 1u << (k % RESCCL_TMA_STAGES);
         hc = (hc & ~(1u << slot)) | (((Lcpar & rb) ? 1u : 0u) << slot);
         Lcpar ^= rb;
@@ -960,9 +1004,14 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
         const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + lj;
         const char* bsrc = (F & kDirect) ? pR + lo_l * T::kSize + off
                                          : pin + (in_seq % RESCCL_K) * RESCCL_SLOT + off;
-        mbar_expect_tx(Lfull + 8 * s, 2 * nb);
-        tma_load(sa, pA + lo_l * T::kSize + off, nb, Lfull + 8 * s, pol_first);
-        tma_load(sa + (u32)RESCCL_TMA_TILE, bsrc, nb, Lfull + 8 * s, pol_first);
+        if (bred) {  // incoming tile only; the local operand is added in L2 by the store
+          mbar_expect_tx(Lfull + 8 * s, nb);
+          tma_load(sa, bsrc, nb, Lfull + 8 * s, pol_first);
+        } else {
+          mbar_expect_tx(Lfull + 8 * s, 2 * nb);
+          tma_load(sa, pA + lo_l * T::kSize + off, nb, Lfull + 8 * s, pol_first);
+          tma_load(sa + (u32)RESCCL_TMA_TILE, bsrc, nb, Lfull + 8 * s, pol_first);
+        }
       } else {
         const char* src;
         if (Kind<F>::has_b) {  // staged receive: the FIFO slot
@@ -980,7 +1029,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       prog = true;
     }
 #if !RESCCL_RING
-    if ((F & kReduce) && published != issued) {  // one word per batch of issued tiles
+    if ((F & kReduce) && !bred && published != issued) {  // one word per batch of issued tiles
       sts_u64(Lqprog, ((u64)ebase << 32) | (u64)(k0 + issued));
       published = issued;
     }
@@ -989,18 +1038,21 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
     while (stored < issued) {
       const u32 slot = stored % P;
       const u32 s = RESCCL_HS(slot);
-      const bool ok = (F & kReduce) ? mbar_test(Lcomp + 8 * s, (hc >> slot) & 1)
-                                    : mbar_test(Lfull + 8 * s, (hf >> slot) & 1);
+      const bool ok = ((F & kReduce) && !bred) ? mbar_test(Lcomp + 8 * s, (hc >> slot) & 1)
+                                               : mbar_test(Lfull + 8 * s, (hf >> slot) & 1);
       if (!ok) break;
       while (st >= T_s) {
         ++sj;
         st = 0;
-        T_s = mb_tiles_m<F>(aM, aMi, plen, sj, Linst, T::kSize, lo_s, nb_s);
+        T_s = mb_tiles_m<F>(aM, aMi, plen, sj, Linst, T::kSize, lo_s, nb_s, bred);
       }
       const i64 off = (i64)st * TB;
       const u32 nb = (u32)((nb_s - off) < TB ? (nb_s - off) : TB);
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
-      if (F & kStore) tma_store(pD1 + lo_s * T::kSize + off, sa, nb, pol_first);
+      if (F & kStore) {
+        if ((F & kReduce) && bred) tma_reduce<T, OP>(pD1 + lo_s * T::kSize + off, sa, nb, pol_first);
+        else tma_store(pD1 + lo_s * T::kSize + off, sa, nb, pol_first);
+      }
       if (Kind<F>::send_data) {
         if (F & kDirect) {
           tma_store(pQ + lo_s * T::kSize + off, sa, nb, pol_first);
@@ -1039,7 +1091,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       post_mb<F>(a, d, p, pj);
       ++pj;
       if (pj < nmb) {
-        T_p = mb_tiles_m<F>(aM, aMi, plen, pj, Linst, T::kSize, lo_p, nb_p);
+        T_p = mb_tiles_m<F>(aM, aMi, plen, pj, Linst, T::kSize, lo_p, nb_p, bred);
         gp_end += T_p;
       }
       prog = true;
@@ -1073,7 +1125,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
         // event the store step needs) instead of polling
         const u32 slot = stored % P;
         const u32 s = RESCCL_HS(slot);
-        if (F & kReduce) (void)mbar_try(Lcomp + 8 * s, (hc >> slot) & 1);
+        if ((F & kReduce) && !bred) (void)mbar_try(Lcomp + 8 * s, (hc >> slot) & 1);
         else (void)mbar_try(Lfull + 8 * s, (hf >> slot) & 1);
         ++spins;
       } else if (++spins > 32) {
@@ -1118,6 +1170,14 @@ __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const Prim
   const i64 aM = a.M, aMi = a.Mi, plen = p.len;
   volatile int* const abort_flag = L.abort_flag;
   u32 k = L.tseq;
+  if (bulk_reduce_prim<T, OP, F>(p.A, p.D1)) {  // the leader adds in L2: only keep the tile count
+    for (int j = 0; j < nmb; ++j) {
+      i64 lo, nbj;
+      k += mb_tiles_m<F>(aM, aMi, plen, j, Linst, T::kSize, lo, nbj, true);
+    }
+    L.tseq = k;
+    return true;
+  }
 #if !RESCCL_RING
   u32 cbase = 0xFFFFFFFFu, cmask = 0, cpar = 0, cR = 1, ci = 0, cu = 0;  // cached epoch, position of k
 #endif

@@ -59,6 +59,7 @@ struct CodegenOpts {
   int prefetch = 0;              // micro-batches of local operand prefetched into L2 ahead (off: r01)
   int pool_cap = 0;              // stages of the CTA pool one lane may hold (0 = all)
   int ring = 0;                  // lane-private stage rings instead of the shared CTA pool
+  int bulkred = 0;               // in-place reduces: bulk-add the incoming tile in L2
   int cpoll = 0;                 // combine warps: 1 = one polling warp + named barrier
   int store_lag = 1;             // bulk stores a lane lets drain before it blocks to reuse a stage
   int exit_barrier = 0;          // direct transport across processes: a rank's kernel ends only

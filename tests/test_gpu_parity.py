@@ -296,3 +296,22 @@ def test_count_2pow24_plus_3_direct_allreduce():
     outs, _, err = run_virtual(R, text, "allreduce", xs, dtype, count)
     assert err == 0
     _check_bytes(outs, definition.allreduce(xs, dtype), "allreduce", n, count)
+
+
+@pytest.mark.parametrize("coll", ["allreduce", "reducescatter"])
+@pytest.mark.parametrize("dtype,op", [("bfloat16", "sum"), ("float32", "sum"), ("int32", "sum"),
+                                      ("float16", "max"), ("float32", "max")])
+@pytest.mark.parametrize("bulkred", [0, 1])
+def test_inplace_tma_reduce_paths(coll, dtype, op, bulkred):
+    """In-place reduce primitives on the TMA engine, with the combine warps (bulkred=0) or
+    the L2 bulk reduction of the incoming tile (bulkred=1; f32 max keeps the combine path):
+    bytes = the oracle's replay (one correctly rounded local (+) incoming per hop, R8)."""
+    n = 8
+    g = oir.generate("ring", coll, n)
+    count = 40000 + 37
+    text = _hdr(g, chunkbytes=1 << 20, instances=2, direct=1, tmamin=4096, bulkred=bulkred)
+    xs = _inputs(coll, dtype, n, count, seed=8)
+    outs, _, err = run_virtual(R, text, coll, xs, dtype, count, op=op, inplace=True)
+    assert err == 0
+    exp = oracle_expect(g, xs, dtype, count, op=op, chunk_bytes=1 << 20, instances=2)
+    _check_bytes(outs, exp, coll, n, count)

@@ -32,6 +32,8 @@ cnt = S // 2  # AR: count; AG: total output; RS: total input (nccl-tests S)
 sn, rn = {"allreduce": (cnt, cnt), "allgather": (cnt // N, cnt), "reducescatter": (cnt, cnt // N)}[COLL]
 s = [(torch.rand(sn, device="cuda:0") * 2 - 1).to(torch.bfloat16) for _ in range(N)]
 r = [torch.empty(rn, device="cuda:0", dtype=torch.bfloat16) for _ in range(N)]
+if os.environ.get("SMB_INPLACE") == "1":  # in-place (AllReduce: recv = send; RS: recv inside send)
+    r = [s[k] if COLL == "allreduce" else s[k][k * rn:(k + 1) * rn] for k in range(N)]
 # algorithmic HBM bytes per rank (direct transport): AR 5(N-1)/N S, RS 3(N-1)/N S, AG 2(N-1)/N S
 HB = {"allreduce": 5.0, "reducescatter": 3.0, "allgather": 2.0}[COLL]
 BUSF = {"allreduce": 2.0 * (N - 1) / N}.get(COLL, (N - 1) / N)
@@ -68,6 +70,7 @@ for geo in GEOS:
                               "sms": min(n_sm, blocks),
                               "S": S, "us": round(ms * 1e3, 1), "busbw_gbs": round(bus, 1),
                               "hbm_gbs": round(hbm, 1), "per_sm_hbm_gbs": round(hbm / min(n_sm, blocks), 1),
-                              "opts": EXTRA, "err": grp.async_error()}), flush=True)
+                              "opts": EXTRA, "inplace": os.environ.get("SMB_INPLACE") == "1",
+                              "err": grp.async_error()}), flush=True)
         finally:
             grp.destroy()
