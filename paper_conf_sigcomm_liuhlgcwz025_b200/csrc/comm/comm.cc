@@ -765,8 +765,15 @@ void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t
   if (elt_size(dt) == 0) fail(rescclInvalidArgument, "bad dtype");
   if ((int)op < 0 || (int)op > 2) fail(rescclInvalidArgument, "bad op");
   if (count > 0 && (!send || !recv)) fail(rescclInvalidArgument, "null buffer");
-  rescclAlgo* algo = ensure_algo(comm, (Coll)coll);
   cudaStream_t s = (cudaStream_t)stream;
+  {
+    // flag epochs (micro-batch bases, exit-barrier and NVLS arrival counts) advance on the
+    // host per call, so a captured launch would replay stale epochs and hang
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone)
+      fail(rescclInvalidUsage, "collectives cannot be captured into CUDA graphs (host-side flag epochs)");
+  }
+  rescclAlgo* algo = ensure_algo(comm, (Coll)coll);
   if (comm->mode != 1) {
     if (count == 0) return;
     if (algo->s->opt.nvls && try_nvls(comm, *algo->s, coll, send, recv, count, dt, op, s)) return;

@@ -315,3 +315,29 @@ def test_inplace_tma_reduce_paths(coll, dtype, op, bulkred):
     assert err == 0
     exp = oracle_expect(g, xs, dtype, count, op=op, chunk_bytes=1 << 20, instances=2)
     _check_bytes(outs, exp, coll, n, count)
+
+
+def test_graph_capture_is_rejected_cleanly():
+    """Flag epochs advance on the host per call, so stream capture is refused with
+    InvalidUsage (instead of a graph whose replays would wait on stale epochs)."""
+    import torch
+    from gpu_helpers import to_torch
+    n, count = 2, 4096
+    grp = R.VirtualGroup(n, 0)
+    try:
+        grp.load(oir.generate("ring", "allreduce", n).to_text())
+        xs = _inputs("allreduce", "float32", n, count)
+        s = [to_torch(x, "float32") for x in xs]
+        r = [torch.empty_like(t) for t in s]
+        st = torch.cuda.Stream()
+        g = torch.cuda.CUDAGraph()
+        with pytest.raises(R.ResCCLError) as e:
+            with torch.cuda.graph(g, stream=st):
+                grp.allreduce(s, r)
+        assert e.value.code == R.rescclInvalidUsage
+    finally:
+        grp.destroy()
+    # the communicator stays usable afterwards
+    outs, _, err = run_virtual(R, oir.generate("ring", "allreduce", n).to_text(), "allreduce", xs, "float32", count)
+    assert err == 0
+    _check_bytes(outs, definition.allreduce(xs, "float32"), "allreduce", n, count)
