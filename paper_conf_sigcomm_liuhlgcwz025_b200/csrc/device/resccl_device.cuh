@@ -824,7 +824,7 @@ __device__ __forceinline__ u32 mb_tiles(const KArgs& a, i64 len, int j, int inst
 // completed.  It never blocks on a remote condition while it holds unposted work, so
 // the pipeline adds no wait edge beyond those of the blocking model (deadlock freedom
 // carries over from the plan check).
-template <class T, int OP, int F>
+template <class T, int OP, int F, bool BRED>
 __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
   const KArgs& a = *L.a;
   // Everything the loop reads per tile lives in registers: the lane, the arguments and
@@ -842,7 +842,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   char* const pin = p.in_data;
   char* const pout = p.out_data;
   const u32 P = RESCCL_POOL;  // slots of the per-tile register records (>= stages held)
-  const bool bred = bulk_reduce_prim<T, OP, F>(pA, pD1);
+  constexpr bool bred = BRED;  // (a template parameter: the per-tile loop stays branch-free)
   const i64 TB = tile_bytes<F>(bred);
   const int nmb = a.n_mb;
   const u32 k0 = L.tseq;
@@ -1369,7 +1369,9 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
   const unsigned long long al =
       (unsigned long long)p.A | (unsigned long long)p.D1 | (unsigned long long)p.R | (unsigned long long)p.Q;
   if ((al & 15) == 0 && a.Mi * T::kSize >= RESCCL_TMA_MIN) {
-    if (L.tid == 0) return pipe_leader<T, OP, F>(L, d, p);
+    if (L.tid == 0)
+      return bulk_reduce_prim<T, OP, F>(p.A, p.D1) ? pipe_leader<T, OP, F, RESCCL_BULKRED != 0>(L, d, p)
+                                                   : pipe_leader<T, OP, F, false>(L, d, p);
     if (L.tid < 32) return true;
     if (F & kReduce) return pipe_compute<T, OP, F>(L, d, p, L.tid - 32, L.nthreads - 32);
     // combine warps only keep the lane's tile counter in step for copy primitives
