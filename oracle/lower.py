@@ -28,9 +28,11 @@ TEST INFRASTRUCTURE ONLY.
 * Buffer mapping (R18, in-place IR, out-of-place execution): a read of <r,c>
   before the first write of <r,c> reads the caller's send buffer; later reads and
   all writes use the receive buffer, except ReduceScatter chunks c != r, which
-  live in a comm-owned scratch buffer.  Output locations never written on r get a
-  local copy primitive (AllGather's own chunk, N = 1) at the head of CTA 0's recv
-  lane.
+  live in a comm-owned scratch buffer.  An output location never written on r
+  (AllGather's own chunk) is stored locally by the first send that moves it out of the
+  send buffer (``store`` on a send / dsend: one read feeds the peer and the local copy);
+  only when no such send exists (N = 1) does it get a copy primitive at the head of
+  CTA 0's recv lane.
 """
 from __future__ import annotations
 
@@ -294,6 +296,14 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
             written = {c for (rr, c) in first_w if rr == r}
             for c in range(ir.nchunks):
                 if is_output(coll, r, c) and c not in written:
+                    # the first data-moving send of the location from the send buffer also
+                    # stores it locally; else a separate copy primitive (module docstring)
+                    first = next((p for p in keep if p.chunk == c and p.kind in ("send", "dsend")
+                                  and p.src_buf == "send"), None)
+                    if first is not None:
+                        first.store = True
+                        first.dst_buf = "recv"
+                        continue
                     cp = Prim(r, "copy", c, -1, src_buf="send", dst_buf="recv", cta=0, lane="R")
                     copies.append(cp)
             final_list = copies + keep

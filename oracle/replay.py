@@ -380,6 +380,9 @@ def replay(plan: Plan, inputs: List[np.ndarray], dtype: str, count: int, op: str
             o = g.chunk_off(p.src_buf, p.chunk)
             d, od = tasks[p.send_task].dst, g.chunk_off(p.rem_out, p.chunk)
             bufs[d][p.rem_out][od + lo:od + hi] = bufs[r][p.src_buf][o + lo:o + hi]
+            if p.kind == "dsend" and p.store:         # ... and the local copy of an unwritten output
+                od2 = g.chunk_off(p.dst_buf, p.chunk)
+                bufs[r][p.dst_buf][od2 + lo:od2 + hi] = bufs[r][p.src_buf][o + lo:o + hi]
             return None
         if p.kind in ("psend", "drecv", "drecv_p"):   # flags only
             return None
@@ -388,6 +391,9 @@ def replay(plan: Plan, inputs: List[np.ndarray], dtype: str, count: int, op: str
             incoming = bufs[s_][p.rem_buf][os_ + lo:os_ + hi].copy()
         if p.recv_task is None:                       # plain send
             o = g.chunk_off(p.src_buf, p.chunk)
+            if p.store:                               # ... storing an unwritten output locally too
+                od2 = g.chunk_off(p.dst_buf, p.chunk)
+                bufs[r][p.dst_buf][od2 + lo:od2 + hi] = bufs[r][p.src_buf][o + lo:o + hi]
             return bufs[r][p.src_buf][o + lo:o + hi].copy()
         if p.reduce:
             o = g.chunk_off(p.src_buf, p.chunk)
@@ -475,6 +481,8 @@ def happens_before_races(plan: Plan, n_mb: int = 2, instances: int = 1, K: int =
             if not (push_recv and phase == 0):
                 acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
                 acc.append(((tasks[p.send_task].dst, p.rem_out, p.chunk, jj, inst), True))
+                if p.kind == "dsend" and p.store and not inplace:  # local copy of an unwritten output
+                    acc.append(((r, p.dst_buf, p.chunk, jj, inst), True))
         elif p.kind in ("prrc", "prrc_p", "prrc_d"):
             acc.append(((tasks[p.recv_task].src, p.rem_buf, p.chunk, jj, inst), False))
             acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
@@ -489,6 +497,8 @@ def happens_before_races(plan: Plan, n_mb: int = 2, instances: int = 1, K: int =
             if p.src_buf and (p.recv_task is None or p.reduce):
                 acc.append(((r, p.src_buf, p.chunk, jj, inst), False))
             if p.recv_task is not None and p.store:
+                acc.append(((r, p.dst_buf, p.chunk, jj, inst), True))
+            if p.recv_task is None and p.store and not inplace:  # send storing an unwritten output
                 acc.append(((r, p.dst_buf, p.chunk, jj, inst), True))
         if inplace and p.kind == "copy":
             acc = []  # in-place, the output already holds the input: the copy does nothing

@@ -1049,7 +1049,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       const i64 off = (i64)st * TB;
       const u32 nb = (u32)((nb_s - off) < TB ? (nb_s - off) : TB);
       const u32 sa = sbase + s * 2 * (u32)RESCCL_TMA_TILE;
-      if (F & kStore) {
+      if ((F & kStore) && pD1) {
         if ((F & kReduce) && bred) tma_reduce<T, OP>(pD1 + lo_s * T::kSize + off, sa, nb, pol_first);
         else tma_store(pD1 + lo_s * T::kSize + off, sa, nb, pol_first);
       }
@@ -1336,6 +1336,9 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
     p.A = buf_ptr(a, L.rank, d.src_buf) + chunk_off<RESCCL_COLL>(d.src_buf, c, a.C) * T::kSize;
   if ((F & kCopy) || (F & kStore))
     p.D1 = buf_ptr(a, L.rank, d.dst_buf) + chunk_off<RESCCL_COLL>(d.dst_buf, c, a.C) * T::kSize;
+  // a send storing an unwritten output locally (AllGather's own chunk): in place the
+  // output already holds it
+  if ((F & kSend) && (F & kStore) && !(F & kRecv) && p.A == p.D1) p.D1 = nullptr;
   if (F & kCopy) {
     if (p.A == p.D1) return true;  // in-place: own chunk already in place
     for (int j = 0; j < a.n_mb; ++j) {

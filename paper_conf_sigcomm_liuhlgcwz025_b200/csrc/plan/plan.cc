@@ -307,11 +307,27 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
         a.dst_buf = BufNone;
       }
     }
-    // final prim list: copies first, then all non-absorbed prims in raw order
+    // final prim list: copies first, then all non-absorbed prims in raw order.  An output
+    // location never written on r (AllGather's own chunk) is copied by the first
+    // data-moving send of it from the send buffer -- it stores its tile locally too (one
+    // read, overlapped with the ring) -- else by a separate copy primitive.  Nothing reads
+    // that location from the receive buffer during the collective, so when the copy
+    // lands does not matter.
     std::vector<Prim> fin;
     std::vector<int> raw_of;  // final index -> raw id (-1 for copies)
     for (int c = 0; c < ir.nchunks; ++c)
       if (is_output(ir.coll, r, c) && !written.count({r, c})) {
+        bool folded = false;
+        for (int i = 0; i < (int)ps.size() && !folded; ++i) {
+          Prim& q = ps[i];
+          if (fused_into.count(i) || q.chunk != c || !(q.flags & kSend) || (q.flags & kRecv) ||
+              (q.flags & kSendPull) || q.src_buf != BufSend)
+            continue;
+          q.flags |= kStore;
+          q.dst_buf = BufRecv;
+          folded = true;
+        }
+        if (folded) continue;
         Prim cp;
         cp.flags = kCopy;
         cp.chunk = c;
