@@ -407,13 +407,25 @@ RDEV_F32(OpSum) RDEV_F32(OpMax) RDEV_F32(OpMin)
 #define RDEV_BF(OPV) \
   template <> __device__ __forceinline__ u32 combine_w<TBF16, OPV>(u32 a, u32 b) { \
     return pack_bf16x2(fop<OPV>(bf_lo(a), bf_lo(b)), fop<OPV>(bf_hi(a), bf_hi(b))); }
-RDEV_BF(OpSum) RDEV_BF(OpMax) RDEV_BF(OpMin)
+RDEV_BF(OpMax) RDEV_BF(OpMin)
 #undef RDEV_BF
 #define RDEV_H(OPV) \
   template <> __device__ __forceinline__ u32 combine_w<TF16, OPV>(u32 a, u32 b) { \
     return pack_f16x2(fop<OPV>(h_lo(a), h_lo(b)), fop<OPV>(h_hi(a), h_hi(b))); }
-RDEV_H(OpSum) RDEV_H(OpMax) RDEV_H(OpMin)
+RDEV_H(OpMax) RDEV_H(OpMin)
 #undef RDEV_H
+// 16-bit sums: one packed add, correctly rounded (RN, subnormals kept) -- the value R8
+// fixes (binary32 add then RNE equals the correctly rounded 16-bit add)
+template <> __device__ __forceinline__ u32 combine_w<TBF16, OpSum>(u32 a, u32 b) {
+  u32 r;
+  asm("add.rn.bf16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+template <> __device__ __forceinline__ u32 combine_w<TF16, OpSum>(u32 a, u32 b) {
+  u32 r;
+  asm("add.rn.f16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
 
 template <class T, int OP>
 __device__ __forceinline__ V4 combine_v(const V4& a, const V4& b) {

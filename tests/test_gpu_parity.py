@@ -341,3 +341,31 @@ def test_graph_capture_is_rejected_cleanly():
     outs, _, err = run_virtual(R, oir.generate("ring", "allreduce", n).to_text(), "allreduce", xs, "float32", count)
     assert err == 0
     _check_bytes(outs, definition.allreduce(xs, "float32"), "allreduce", n, count)
+
+
+@pytest.mark.parametrize("dtype", ["bfloat16", "float16"])
+@pytest.mark.parametrize("tma", [0, 1])
+def test_16bit_add_all_bit_patterns(dtype, tma):
+    """Packed 16-bit adds (add.rn.bf16x2 / add.rn.f16x2) against the correctly rounded sum
+    on (almost) every finite bit pattern -- subnormals, ties, signed zeros included: two
+    ranks, one add per element, so the definition's single rounding is the exact answer."""
+    import numpy as np
+    n = 2
+    pats = np.arange(1 << 16, dtype=np.uint32).astype(np.uint16)
+    if dtype == "bfloat16":
+        f = numerics.bf16_to_f32(pats)
+    else:
+        f = pats.view(np.float16).astype(np.float32)
+    keep = np.isfinite(f) & (np.abs(f) < (2.0 ** 100 if dtype == "bfloat16" else 16384.0))
+    a = pats[keep]
+    rng = np.random.default_rng(11)
+    b = a[rng.permutation(a.size)]
+    xs = [a.copy(), b.copy()]
+    if dtype == "float16":
+        xs = [x.view(np.float16) for x in xs]
+    count = xs[0].size
+    g = oir.generate("ring", "allreduce", n)
+    text = _hdr(g, chunkbytes=1 << 20, instances=2, direct=1, tmamin=4096 if tma else 1 << 30)
+    outs, _, err = run_virtual(R, text, "allreduce", xs, dtype, count)
+    assert err == 0
+    _check_bytes(outs, definition.allreduce(xs, dtype), "allreduce", n, count)
