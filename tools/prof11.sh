@@ -1,0 +1,13 @@
+# final r01 code (bulk reduce, AG fold, packed adds): gpu suite, bench lines, launch list + ncu --set full of the bench kernel
+mkdir -p gpurun_out
+export RESCCL_TIMEOUT_MS=20000
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_v11.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu_v11.log 2>&1; echo "pytest=$?" >> gpurun_out/pytest_gpu_v11.log
+python bench.py > gpurun_out/bench_v11.json 2> gpurun_out/bench_v11.err
+python bench.py --direct 0 --steps 20 --warmup 5 --no-cpu-baseline > gpurun_out/bench_v11_staged.json 2> gpurun_out/bench_v11_staged.err
+ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_v11.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --e2e-steps 0 > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:resccl -s 3 -c 1 -o gpurun_out/prof_ring_ar8_v11 python bench.py --steps 1 --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/ncu_full_v11.log 2>&1
+ncu -i gpurun_out/prof_ring_ar8_v11.ncu-rep --page raw --csv > gpurun_out/prof_v11_raw.csv 2>/dev/null
+ncu -i gpurun_out/prof_ring_ar8_v11.ncu-rep --page details --csv > gpurun_out/prof_v11_details.csv 2>/dev/null
+rm -f gpurun_out/prof_ring_ar8_v11.ncu-rep
+tail -3 gpurun_out/pytest_gpu_v11.log; cat gpurun_out/bench_v11.json
