@@ -58,7 +58,9 @@ def parse():
     p.add_argument("--inplace-steps", type=int, default=10,
                    help="also time in-place calls (recv = send) -> config.inplace_busbw_gbs")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--sweep", default="", help="comma-separated MiB sizes for an extra busBW sweep")
+    p.add_argument("--sweep", default="1,16,64",
+                   help="comma-separated MiB-per-rank sizes for the busBW-vs-size points reported beside the "
+                        "headline (slices of the bench buffers; small points are L2-resident); '' = none")
     return p.parse_args()
 
 
@@ -507,7 +509,7 @@ def main():
         "async_error": err,
     }
     if sweep:
-        line["sweep_busbw_gbs"] = sweep
+        line["sweep_busbw_gbs"] = sweep  # busBW vs size (BASELINE metric); not the headline value
     print(json.dumps(line), flush=True)
     if multi:
         torch.distributed.destroy_process_group()
