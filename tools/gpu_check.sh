@@ -7,3 +7,5 @@ echo "pytest=$?" >> gpurun_out/pytest_gpu.log
 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
 tail -3 gpurun_out/pytest_gpu.log
 cat gpurun_out/bench_default.json
+python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_reference.json 2> gpurun_out/bench_reference.err
+cat gpurun_out/bench_reference.json
