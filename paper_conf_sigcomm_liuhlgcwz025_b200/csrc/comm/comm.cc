@@ -53,6 +53,7 @@ struct KArgs {
   unsigned long long timeout_ns;
   unsigned long long* trace;
   unsigned long long epoch;
+  unsigned long long* epochs;  // device-side epochs {mb_base, epoch, CTAs done}, or null
 };
 
 thread_local std::string g_last_error;
@@ -139,12 +140,13 @@ struct Options {
   int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
   int direct = 0;    // direct transport (R23): virtual ranks / single-process only
   int l2hint = 1;
-  int tma_min = 163840;  // r01: register path wins below ~160 KiB slices (latency-bound)
+  int tma_min = 32768;   // r01 (24 KiB tiles): the TMA engine wins from 32 KiB slices (16 MiB AR +31%)
   int backoff = 1;
   int jitter = 0;
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
   int pool_cap = 0;  // stages of the CTA pool one lane may hold (0 = all)
   int ring = 0;      // lane-private TMA stage rings (1) vs one pool shared by both lanes (0)
+  int devepoch = 1;  // device-side flag epochs (graph-capturable launches) vs host-side (0)
   int bulkred = -1;  // in-place reduce primitives: cp.reduce.async.bulk of the incoming tile
                      // (-1 = auto: on for AllReduce, where it measured +16% per SM; r01_bulkred_inplace)
   int cpoll = 0;     // combine warps: one polling warp + named barrier (1) vs all polling (0)
@@ -201,6 +203,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "ring") o.ring = (int)to_long(v, k);
   else if (k == "cpoll") o.cpoll = (int)to_long(v, k);
   else if (k == "bulkred") o.bulkred = (int)to_long(v, k);
+  else if (k == "devepoch") o.devepoch = (int)to_long(v, k);
   else if (k == "nvls") o.nvls = (int)to_long(v, k);
   else if (k == "nvlsctas") o.nvls_ctas = (int)to_long(v, k);
   else if (k == "sched") {
@@ -223,7 +226,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_BULKRED", "bulkred"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_BULKRED", "bulkred"}, {"RESCCL_DEVEPOCH", "devepoch"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -343,6 +346,7 @@ struct AlgoShared {
   Layout lay;
   std::string json;
   unsigned long long mb_cum = 0;       // virtual group: one counter for all ranks
+  unsigned long long* dev_epochs = nullptr;  // virtual group: device-side epochs (devepoch=1)
   std::map<std::string, Kern> kernels;  // key: dtype/op/ranks/scope
   std::vector<char*> region;           // virtual group: per-rank plan region (one allocation)
   unsigned long long* trace_host = nullptr;  // RESCCL_TRACE buffer (host-mapped)
@@ -362,6 +366,7 @@ struct rescclAlgo {
   unsigned long long mb_cum = 0;       // multi-process: this rank's counter
   unsigned long long twin_mb_cum = 0;  // ... and its staged twin's
   unsigned long long epoch = 0;        // direct calls issued (exit-barrier target)
+  unsigned long long* dev_epochs[2] = {nullptr, nullptr};  // multi-process: device epochs (plan, twin)
 };
 
 namespace {
@@ -476,7 +481,7 @@ std::string info_json(const AlgoShared& a) {
   o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
     << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"tma\":" << a.opt.tma
     << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"l2hint\":" << a.opt.l2hint << ",\"prefetch\":" << a.opt.prefetch << ",\"sched\":\""
-    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"bulkred\":" << a.opt.bulkred << ",\"nvls\":" << a.opt.nvls << ",\"nvlsctas\":" << a.opt.nvls_ctas << ",\"linkmodel\":\""
+    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"bulkred\":" << a.opt.bulkred << ",\"devepoch\":" << a.opt.devepoch << ",\"nvls\":" << a.opt.nvls << ",\"nvlsctas\":" << a.opt.nvls_ctas << ",\"linkmodel\":\""
     << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
     << ",\"ctas\":[";
   for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];
@@ -699,6 +704,7 @@ void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const vo
   ka.err = comm->err_dev;
   ka.timeout_ns = timeout_ns();
   ka.trace = trace_buffer(a, a.lay.ctas[comm->rank] * a.opt.instances, ka.block_base);
+  if (a.opt.devepoch) ka.epochs = algo->dev_epochs[ap == algo->s.get() ? 0 : 1];
   const bool use_tma = a.opt.tma && g.Mi * elt_size(c.dt) >= a.opt.tma_min;
   Kern& k = get_kernel(a, c.dt, c.op, comm->rank, comm->rank + 1, false, use_tma);
   launch(k, a.lay.ctas[comm->rank] * a.opt.instances, 32 * a.opt.nwarps, ka, s);
@@ -729,6 +735,7 @@ void group_launch(Group* G, Pending& p) {
   ka.err = G->err_dev;
   ka.timeout_ns = timeout_ns();
   ka.trace = trace_buffer(a, a.lay.total_pairs * a.opt.instances, 0);
+  if (a.opt.devepoch) ka.epochs = a.dev_epochs;
   const bool use_tma = a.opt.tma && g.Mi * elt_size(c.dt) >= a.opt.tma_min;
   Kern& k = get_kernel(a, c.dt, c.op, 0, G->nranks, true, use_tma);
   cudaStream_t ls = p.streams.back();
@@ -766,14 +773,18 @@ void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t
   if ((int)op < 0 || (int)op > 2) fail(rescclInvalidArgument, "bad op");
   if (count > 0 && (!send || !recv)) fail(rescclInvalidArgument, "null buffer");
   cudaStream_t s = (cudaStream_t)stream;
-  {
-    // flag epochs (micro-batch bases, exit-barrier and NVLS arrival counts) advance on the
-    // host per call, so a captured launch would replay stale epochs and hang
-    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-    if (cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone)
-      fail(rescclInvalidUsage, "collectives cannot be captured into CUDA graphs (host-side flag epochs)");
-  }
+  // CUDA-graph capture: the generated kernels take their flag epochs from device memory
+  // (devepoch=1, default), so a captured launch replays correctly; host-side epochs
+  // (devepoch=0) and the NVLS transport's arrival counts advance on the host per call, so
+  // those refuse capture rather than build a graph whose replays would hang
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  const bool capturing = cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone;
+  if (capturing && !comm->active[coll])
+    fail(rescclInvalidUsage, "load an algorithm before capturing a collective into a CUDA graph");
   rescclAlgo* algo = ensure_algo(comm, (Coll)coll);
+  if (capturing && (!algo->s->opt.devepoch || algo->s->opt.nvls))
+    fail(rescclInvalidUsage, "this algorithm cannot be captured into a CUDA graph (devepoch=0 or nvls=1: "
+                             "host-side epochs)");
   if (comm->mode != 1) {
     if (count == 0) return;
     if (algo->s->opt.nvls && try_nvls(comm, *algo->s, coll, send, recv, count, dt, op, s)) return;
@@ -810,6 +821,16 @@ void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t
   }
 }
 
+// device-side epochs {mb_base, epoch, CTAs done}, zeroed (freed with the communicator)
+unsigned long long* alloc_epochs(int dev) {
+  cuda_check(cudaSetDevice(dev), "cudaSetDevice");
+  unsigned long long* p = nullptr;
+  cuda_check(cudaMalloc((void**)&p, 4 * sizeof(unsigned long long)), "cudaMalloc(epochs)");
+  cuda_check(cudaMemset(p, 0, 4 * sizeof(unsigned long long)), "cudaMemset(epochs)");
+  cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
+  return p;
+}
+
 // ---------------------------------------------------------------- algorithm loading
 rescclAlgo* load_algo(rescclComm* comm, const std::string& text) {
   std::shared_ptr<AlgoShared> s;
@@ -826,6 +847,7 @@ rescclAlgo* load_algo(rescclComm* comm, const std::string& text) {
       cuda_check(cudaMemset(s->region_alloc, 0, bytes), "cudaMemset(region)");
       cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
       for (int q = 0; q < G->nranks; ++q) s->region.push_back(s->region_alloc + (size_t)q * s->lay.region_bytes);
+      s->dev_epochs = alloc_epochs(G->dev);
       G->algos[text] = s;
     }
   } else {
@@ -848,6 +870,10 @@ rescclAlgo* load_algo(rescclComm* comm, const std::string& text) {
   auto algo = std::make_unique<rescclAlgo>();
   algo->s = s;
   algo->comm = comm;
+  if (comm->mode != 1) {  // this rank's device-side epochs for the plan and its staged twin
+    algo->dev_epochs[0] = alloc_epochs(comm->dev);
+    if (s->twin) algo->dev_epochs[1] = alloc_epochs(comm->dev);
+  }
   rescclAlgo* raw = algo.get();
   comm->algos.push_back(std::move(algo));
   comm->active[(int)s->ir.coll] = raw;
@@ -1448,6 +1474,7 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
           if (k.second.mod) driver().ModuleUnload(k.second.mod);
         kv.second->kernels.clear();
         if (kv.second->region_alloc) cudaFree(kv.second->region_alloc);
+        if (kv.second->dev_epochs) cudaFree(kv.second->dev_epochs);
       }
       for (auto e : G->events) cudaEventDestroy(e);
       cudaFreeHost(G->err_host);
@@ -1457,6 +1484,8 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
     }
   } else {
     for (auto& a : comm->algos) {
+      for (auto* e : a->dev_epochs)
+        if (e) cudaFree(e);
       if (a->s.use_count() == 1)
         for (AlgoShared* x : {a->s.get(), a->s->twin.get()})
           if (x)
