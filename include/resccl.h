@@ -17,7 +17,12 @@
  *  - In-place: AllReduce sendbuf == recvbuf; AllGather sendbuf == recvbuf +
  *    rank*sendcount*size; ReduceScatter recvbuf == sendbuf + rank*recvcount*size.
  *  - Collective calls only enqueue work on `stream` (cudaStream_t passed as void*;
- *    NULL = legacy default stream); they never synchronise the device.
+ *    NULL = legacy default stream); they never synchronise the device.  They may be
+ *    captured into CUDA graphs: the generated kernels read their flag epochs from device
+ *    memory and advance them themselves (header option devepoch=1, the default), so graph
+ *    replays and eager calls of the same algorithm interleave freely.  devepoch=0 and
+ *    nvls=1 keep host-side epochs and refuse capture (InvalidUsage); load the algorithm
+ *    before capturing (loading allocates).
  *  - All ranks issue the same collectives in the same order with the same count,
  *    dtype and op; a communicator is not thread-safe.
  *  - Every function returns a rescclResult_t; no exception crosses the ABI and the

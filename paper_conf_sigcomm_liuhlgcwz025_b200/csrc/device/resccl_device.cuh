@@ -57,7 +57,38 @@ struct KArgs {
   u64 timeout_ns;
   u64* trace;                         // RESCCL_TRACE: 4 x u64 per (block, lane), host-mapped
   u64 epoch;                          // RESCCL_EXIT_BARRIER: calls of this plan issued before
+  u64* epochs;                        // device-side epochs (graph-capturable launches), or null:
+                                      // {mb_base, epoch, CTAs done}; the kernel reads the first two
+                                      // instead of the fields above, the last CTA advances them
 };
+
+// Device-side epochs: every CTA takes this launch's micro-batch base and call epoch from
+// device memory (so a CUDA graph replays with fresh epochs); the last CTA to finish
+// advances them by this call's micro-batches / one call.  Stream order makes the update
+// visible to the next launch of the plan.
+__device__ __forceinline__ const KArgs* epochs_begin(const KArgs& a, KArgs* sh) {
+  if (!a.epochs) return &a;
+  if (threadIdx.x == 0) {
+    *sh = a;
+    sh->mb_base = *(volatile u64*)&a.epochs[0];
+    sh->epoch = *(volatile u64*)&a.epochs[1];
+  }
+  __syncthreads();
+  return sh;
+}
+__device__ __forceinline__ void epochs_end(const KArgs& a) {
+  if (!a.epochs) return;
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  __threadfence();
+  const unsigned long long old = atomicAdd((unsigned long long*)&a.epochs[2], 1ull);
+  if (old == (unsigned long long)gridDim.x - 1) {
+    a.epochs[0] += (u64)a.n_mb;
+    a.epochs[1] += 1;
+    a.epochs[2] = 0;
+    __threadfence();
+  }
+}
 
 enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16, kDirect = 32, kPull = 64, kSendPull = 128 };
 enum : int { BufNone = -1, BufSend = 0, BufRecv = 1, BufScratch = 2 };
@@ -1377,7 +1408,7 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
   // no data moved here: pull-send, push-receive (+ readable for the next hop)
   if ((F & kDirect) && !Kind<F>::has_b && !Kind<F>::send_data) return L.tid == 0 ? run_flags<F>(L, d, p) : true;
 #ifndef RESCCL_TMA_MIN
-#define RESCCL_TMA_MIN 163840
+#define RESCCL_TMA_MIN 32768
 #endif
 #if RESCCL_TMA
   // small slices are latency-bound: the register path saves two bulk-copy round trips

@@ -53,7 +53,7 @@ struct CodegenOpts {
   int tma_stages = 2;            // stages per lane (the CTA pool holds 2x)
   int trace = 0;                 // per-lane lifetime / wait timers (TB utilisation, Table 3)
   int l2hint = 1;                // L2 evict_last on FIFO writes, evict_first on streams
-  int tma_min = 163840;          // slices below this many bytes use the register path
+  int tma_min = 32768;           // slices below this many bytes use the register path
   int backoff = 1;               // nanosleep back-off while polling flags
   int jitter = 0;                // debug fault injector: random delays around every sync
   int prefetch = 0;              // micro-batches of local operand prefetched into L2 ahead (off: r01)

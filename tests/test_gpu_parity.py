@@ -317,15 +317,61 @@ def test_inplace_tma_reduce_paths(coll, dtype, op, bulkred):
     _check_bytes(outs, exp, coll, n, count)
 
 
-def test_graph_capture_is_rejected_cleanly():
-    """Flag epochs advance on the host per call, so stream capture is refused with
-    InvalidUsage (instead of a graph whose replays would wait on stale epochs)."""
+@pytest.mark.parametrize("name,coll,kw", [("ring", "allreduce", {}), ("hm", "allreduce", {"g": 2}),
+                                          ("ring", "allgather", {}), ("dbt", "allreduce", {})])
+@pytest.mark.parametrize("tmamin", [4096, 1 << 30])
+def test_cuda_graph_capture_and_replay(name, coll, kw, tmamin):
+    """Device-side flag epochs (devepoch=1): collectives captured into a CUDA graph replay
+    correctly, interleaved with eager calls of the same plan (the epochs the graph's
+    kernels read advance on the device)."""
+    import torch
+    from gpu_helpers import to_numpy, to_torch
+    n, count, dtype = 4, 30000 + 5, "int32"
+    g = oir.generate(name, coll, n, **kw)
+    text = _hdr(g, chunkbytes=1 << 16, instances=2, direct=1, tmamin=tmamin)
+    grp = R.VirtualGroup(n, 0)
+    try:
+        grp.load(text)
+        ref_in = [_inputs(coll, dtype, n, count, seed=s) for s in (21, 22)]
+        s = [to_torch(x, dtype) for x in ref_in[0]]
+        m = count * n if coll == "allgather" else count
+        r = [torch.zeros(m, dtype=torch.int32, device="cuda:0") for _ in range(n)]
+        f = getattr(grp, coll)
+        f(s, r)  # eager warm-up (compiles the kernel outside the capture)
+        torch.cuda.synchronize()
+        st = torch.cuda.Stream()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=st):
+            f(s, r, stream=st)
+            f(s, r, stream=st)
+        for it in range(3):
+            x = ref_in[it % 2]
+            for t, v in zip(s, x):
+                t.copy_(to_torch(v, dtype))
+            for t in r:
+                t.zero_()
+            graph.replay()
+            torch.cuda.synchronize()
+            assert grp.async_error() == 0
+            outs = [to_numpy(t, dtype) for t in r]
+            _check_bytes(outs, definition_expect(coll, x, dtype), coll, n, count)
+            f(s, r)  # an eager call between replays advances the same epochs
+            torch.cuda.synchronize()
+            _check_bytes([to_numpy(t, dtype) for t in r], definition_expect(coll, x, dtype), coll, n, count)
+    finally:
+        grp.destroy()
+
+
+def test_graph_capture_refused_with_host_epochs():
+    """devepoch=0 keeps host-side epochs: capture is refused with InvalidUsage before any
+    CUDA state changes, and the communicator stays usable."""
     import torch
     from gpu_helpers import to_torch
     n, count = 2, 4096
+    text = _hdr(oir.generate("ring", "allreduce", n), devepoch=0)
     grp = R.VirtualGroup(n, 0)
     try:
-        grp.load(oir.generate("ring", "allreduce", n).to_text())
+        grp.load(text)
         xs = _inputs("allreduce", "float32", n, count)
         s = [to_torch(x, "float32") for x in xs]
         r = [torch.empty_like(t) for t in s]
@@ -337,8 +383,7 @@ def test_graph_capture_is_rejected_cleanly():
         assert e.value.code == R.rescclInvalidUsage
     finally:
         grp.destroy()
-    # the communicator stays usable afterwards
-    outs, _, err = run_virtual(R, oir.generate("ring", "allreduce", n).to_text(), "allreduce", xs, "float32", count)
+    outs, _, err = run_virtual(R, text, "allreduce", xs, "float32", count)
     assert err == 0
     _check_bytes(outs, definition.allreduce(xs, "float32"), "allreduce", n, count)
 
