@@ -218,3 +218,94 @@ def test_ipc_registered_windows_direct(algo, coll, world, count, opts):
         for it, o in enumerate(outs):
             e = exp_s if (it == 1 or coll == "reducescatter") else exp_d
             assert np.array_equal(o.view(np.uint8), e[r].view(np.uint8)), f"rank {r} call {it}"
+
+
+def _graph_worker(rank, world, port, count, q):
+    """Device-side epochs across processes: a CUDA graph of a registered-window (direct,
+    exit barrier) AllReduce and an unregistered (staged twin) one, replayed between eager
+    calls of both plans."""
+    try:
+        import sys
+        root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+        sys.path.insert(0, root)
+        sys.path.insert(0, os.path.join(root, "tests"))
+        import torch
+        import torch.distributed as dist
+        import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+        import resccl_inputs as inp
+        from gpu_helpers import to_numpy, to_torch
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        comm = R.init_process_group_comm(rank, world, 0)
+        text = R.rescclGenerateIr("ring", "allreduce", world)
+        hdr, rest = text.split("\n", 1)
+        comm.load(hdr + " chunkbytes=65536 instances=2 fifodepth=2 direct=1\n" + rest)
+        x = to_torch(inp.rank_input("int32", 9, rank, count), "int32")
+        win = torch.zeros(2 * count + 64, dtype=torch.int32, device="cuda:0")
+        comm.register(win)
+        s_reg, r_reg = win[:count], win[count + 64:2 * count + 64]
+        s_reg.copy_(x)
+        r_un = torch.zeros(count, dtype=torch.int32, device="cuda:0")
+        comm.allreduce(s_reg, r_reg)  # eager warm-up: both plans compiled outside the capture
+        comm.allreduce(x, r_un)
+        torch.cuda.synchronize()
+        dist.barrier()
+        st = torch.cuda.Stream()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            comm.allreduce(s_reg, r_reg, stream=st)
+            comm.allreduce(x, r_un, stream=st)
+        outs = []
+        for it in range(3):
+            r_reg.zero_()
+            r_un.zero_()
+            torch.cuda.synchronize()
+            dist.barrier()
+            g.replay()
+            torch.cuda.synchronize()
+            outs.append((to_numpy(r_reg.clone(), "int32"), to_numpy(r_un.clone(), "int32")))
+            dist.barrier()
+            comm.allreduce(s_reg, r_reg)  # eager calls advance the same device epochs
+            comm.allreduce(x, r_un)
+            torch.cuda.synchronize()
+            outs.append((to_numpy(r_reg.clone(), "int32"), to_numpy(r_un.clone(), "int32")))
+        err = comm.async_error()
+        dist.barrier()
+        comm.destroy()
+        dist.destroy_process_group()
+        q.put((rank, outs, err, None))
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put((rank, None, None, traceback.format_exc()))
+
+
+@pytest.mark.timeout(300)
+def test_ipc_cuda_graph_replay_device_epochs():
+    import torch.multiprocessing as mp
+    import resccl_inputs as inp
+    from oracle import definition
+    world, count = 2, 50000 + 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    os.environ["RESCCL_TIMEOUT_MS"] = "120000"
+    procs = [ctx.Process(target=_graph_worker, args=(r, world, port, count, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        rank, outs, err, tb = q.get(timeout=280)
+        assert tb is None, tb
+        res[rank] = (outs, err)
+    for p in procs:
+        p.join(30)
+    xs = [inp.rank_input("int32", 9, r, count) for r in range(world)]
+    exp = definition.allreduce(xs, "int32")
+    for r in range(world):
+        outs, err = res[r]
+        assert err == 0
+        for k, (a, b) in enumerate(outs):
+            assert np.array_equal(a, exp[r]), f"rank {r} step {k} (window)"
+            assert np.array_equal(b, exp[r]), f"rank {r} step {k} (twin)"
