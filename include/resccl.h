@@ -23,6 +23,17 @@
  *    replays and eager calls of the same algorithm interleave freely.  devepoch=0 and
  *    nvls=1 keep host-side epochs and refuse capture (InvalidUsage); load the algorithm
  *    before capturing (loading allocates).
+ *  - Host buffers: a collective's sendbuf and/or recvbuf may be host memory (pinned
+ *    for asynchronous copies; pageable works at pageable-copy speed).  The library
+ *    stages it through device memory the communicator owns (grown on demand, freed
+ *    by rescclCommDestroy): uploads on an internal copy stream, the collective on
+ *    `stream`, downloads on a second copy stream, and `stream` waits for the last
+ *    download, so the result is in recvbuf once `stream` completes.  AllReduce is
+ *    cut into pieces of RESCCL_HOST_PIECE bytes (default 32 MiB) whose upload,
+ *    collective and download overlap.  The host in-place rules are the device ones.
+ *    Host-buffer calls refuse CUDA-graph capture (InvalidUsage).  Staged calls of a
+ *    direct=1 algorithm across processes run its staged twin (the stage is not a
+ *    registered window).
  *  - All ranks issue the same collectives in the same order with the same count,
  *    dtype and op; a communicator is not thread-safe.
  *  - Every function returns a rescclResult_t; no exception crosses the ABI and the

@@ -374,6 +374,19 @@ struct Group;
 struct NvlsWin;
 }
 
+// copy streams and events of host-buffer collectives (upload, download)
+struct HostCopy {
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  std::vector<cudaEvent_t> ev;
+  void release() {
+    for (auto e : ev) cudaEventDestroy(e);
+    ev.clear();
+    if (h2d) cudaStreamDestroy(h2d);
+    if (d2h) cudaStreamDestroy(d2h);
+    h2d = d2h = nullptr;
+  }
+};
+
 struct rescclComm {
   int rank = 0, nranks = 1, dev = 0;
   bool connected = false;
@@ -400,6 +413,10 @@ struct rescclComm {
   std::vector<Window> windows;
   std::map<std::string, char*> ipc_maps;  // opened peer allocations (handle bytes -> mapped base)
   std::vector<std::shared_ptr<NvlsWin>> nvls;  // f3: this rank's NVLS windows (multicast-bound)
+  // host-buffer collectives: device staging (send and receive regions) of this rank
+  char* hstage = nullptr;
+  size_t hstage_bytes = 0;
+  HostCopy hcopy;  // host-buffer collectives: copy streams (multi-process / multi-device)
 };
 
 namespace {
@@ -413,6 +430,7 @@ struct Pending {
   std::vector<const void*> send;
   std::vector<void*> recv;
   std::vector<cudaStream_t> streams;
+  bool host = false;  // some rank passed a host buffer (staged by group_host_launch)
 };
 
 struct Group {
@@ -425,6 +443,7 @@ struct Group {
   int* err_host = nullptr;
   int* err_dev = nullptr;
   std::vector<cudaEvent_t> events;
+  HostCopy hcopy;  // host-buffer collectives of the group
   int refs = 0;
 };
 
@@ -761,6 +780,199 @@ void group_launch(Group* G, Pending& p) {
   }
 }
 
+
+// ------------------------------------------------------------ host-buffer collectives
+// A send or receive buffer in host memory (pinned, or pageable at pageable-copy speed) is
+// staged through device memory the communicator owns: upload on a copy stream, the
+// collective on the caller's stream, download on a second copy stream.  AllReduce is cut
+// into pieces of RESCCL_HOST_PIECE bytes (default 32 MiB) so that piece k's collective
+// and piece k-1's download overlap piece k+1's upload (PCIe is full duplex).  The
+// caller's stream waits for the last download: stream semantics are the device path's.
+
+bool host_ptr(const void* p) {
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return true;
+  }
+  return at.type == cudaMemoryTypeHost || at.type == cudaMemoryTypeUnregistered;
+}
+
+size_t host_piece_bytes() {
+  const char* v = getenv("RESCCL_HOST_PIECE");
+  long long b = v ? atoll(v) : (32ll << 20);
+  if (b < 4096) b = 4096;
+  return (size_t)b & ~(size_t)255;
+}
+
+void ensure_hstage(rescclComm* comm, size_t bytes) {
+  if (comm->hstage_bytes >= bytes) return;
+  cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+  if (comm->hstage) {
+    cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");  // queued work may use it
+    cuda_check(cudaFree(comm->hstage), "cudaFree(host stage)");
+    comm->hstage = nullptr;
+    comm->hstage_bytes = 0;
+  }
+  cuda_check(cudaMalloc((void**)&comm->hstage, bytes), "cudaMalloc(host stage)");
+  comm->hstage_bytes = bytes;
+}
+
+void ensure_copy(HostCopy& h, size_t nev) {
+  if (!h.h2d) {
+    cuda_check(cudaStreamCreateWithFlags(&h.h2d, cudaStreamNonBlocking), "cudaStreamCreate");
+    cuda_check(cudaStreamCreateWithFlags(&h.d2h, cudaStreamNonBlocking), "cudaStreamCreate");
+  }
+  while (h.ev.size() < nev) {
+    cudaEvent_t e;
+    cuda_check(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
+    h.ev.push_back(e);
+  }
+}
+
+// One rank's staging: device offsets of the send / receive regions in its stage (-1 =
+// the caller's device buffer).  Host in-place calls (NCCL's rules: AR send == recv, AG
+// send == recv + rank*count, RS recv == send + rank*count) stage one region.
+struct StagePlan {
+  size_t sb = 0, rb = 0, need = 0;
+  long long soff = -1, roff = -1;
+  bool hs = false, hr = false;
+};
+
+StagePlan stage_plan(int coll, int rank, int nranks, const void* send, void* recv, size_t count, size_t e) {
+  StagePlan P;
+  P.sb = count * e * (coll == (int)Coll::ReduceScatter ? nranks : 1);
+  P.rb = count * e * (coll == (int)Coll::AllGather ? nranks : 1);
+  P.hs = host_ptr(send);
+  P.hr = host_ptr(recv);
+  const char* sp = (const char*)send;
+  const char* rp = (const char*)recv;
+  const size_t blk = (size_t)rank * count * e;
+  if (P.hs && P.hr && coll == (int)Coll::AllReduce && sp == rp) {
+    P.need = P.rb, P.soff = P.roff = 0;
+  } else if (P.hs && P.hr && coll == (int)Coll::AllGather && sp == rp + blk) {
+    P.need = P.rb, P.roff = 0, P.soff = (long long)blk;
+  } else if (P.hs && P.hr && coll == (int)Coll::ReduceScatter && rp == sp + blk) {
+    P.need = P.sb, P.soff = 0, P.roff = (long long)blk;
+  } else {
+    if (P.hs) P.soff = 0, P.need += P.sb;
+    if (P.hr) P.roff = (long long)P.need, P.need += P.rb;
+  }
+  return P;
+}
+
+size_t piece_elems(int coll, size_t count, size_t e) {
+  return coll == (int)Coll::AllReduce ? std::min(count, std::max<size_t>(1, host_piece_bytes() / e)) : count;
+}
+
+// multi-process / multi-device rank
+void host_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const void* send, void* recv,
+               cudaStream_t s) {
+  const size_t e = elt_size(c.dt);
+  const StagePlan P = stage_plan(c.coll, comm->rank, comm->nranks, send, recv, c.count, e);
+  ensure_hstage(comm, P.need);
+  const char* ds = P.soff >= 0 ? comm->hstage + P.soff : (const char*)send;
+  char* dr = P.roff >= 0 ? comm->hstage + P.roff : (char*)recv;
+  const size_t pe = piece_elems(c.coll, c.count, e), np = (c.count + pe - 1) / pe;
+  HostCopy& h = comm->hcopy;
+  ensure_copy(h, 2 * np + 2);
+  size_t ei = 0;
+  cuda_check(cudaEventRecord(h.ev[ei], s), "cudaEventRecord");
+  cuda_check(cudaStreamWaitEvent(h.h2d, h.ev[ei], 0), "cudaStreamWaitEvent");
+  cuda_check(cudaStreamWaitEvent(h.d2h, h.ev[ei++], 0), "cudaStreamWaitEvent");
+  for (size_t k = 0; k < np; ++k) {
+    const size_t lo = k * pe, n = std::min(pe, c.count - lo);
+    const size_t off = c.coll == (int)Coll::AllReduce ? lo * e : 0;
+    if (P.hs) {
+      cuda_check(cudaMemcpyAsync((char*)ds + off, (const char*)send + off, c.coll == (int)Coll::AllReduce ? n * e : P.sb,
+                                 cudaMemcpyHostToDevice, h.h2d), "cudaMemcpyAsync(H2D)");
+      cuda_check(cudaEventRecord(h.ev[ei], h.h2d), "cudaEventRecord");
+      cuda_check(cudaStreamWaitEvent(s, h.ev[ei++], 0), "cudaStreamWaitEvent");
+    }
+    launch_rank(comm, algo, CallDesc{c.coll, n, c.dt, c.op}, ds + off, dr + off, s);
+    if (P.hr) {
+      cuda_check(cudaEventRecord(h.ev[ei], s), "cudaEventRecord");
+      cuda_check(cudaStreamWaitEvent(h.d2h, h.ev[ei++], 0), "cudaStreamWaitEvent");
+      cuda_check(cudaMemcpyAsync((char*)recv + off, dr + off, c.coll == (int)Coll::AllReduce ? n * e : P.rb,
+                                 cudaMemcpyDeviceToHost, h.d2h), "cudaMemcpyAsync(D2H)");
+    }
+  }
+  if (P.hr) {
+    cuda_check(cudaEventRecord(h.ev[ei], h.d2h), "cudaEventRecord");
+    cuda_check(cudaStreamWaitEvent(s, h.ev[ei++], 0), "cudaStreamWaitEvent");
+  }
+}
+
+// virtual group: every rank's uploads of piece k, one launch for piece k, its downloads
+void group_host_launch(Group* G, Pending& p) {
+  const int N = G->nranks;
+  const size_t e = elt_size((rescclDataType_t)p.dtype);
+  cuda_check(cudaSetDevice(G->dev), "cudaSetDevice");
+  std::vector<StagePlan> P(N);
+  std::vector<const char*> ds(N);
+  std::vector<char*> dr(N);
+  bool any_hs = false, any_hr = false;
+  for (int q = 0; q < N; ++q) {
+    P[q] = stage_plan(p.coll, q, N, p.send[q], p.recv[q], p.count, e);
+    ensure_hstage(G->comms[q], P[q].need);
+    ds[q] = P[q].soff >= 0 ? G->comms[q]->hstage + P[q].soff : (const char*)p.send[q];
+    dr[q] = P[q].roff >= 0 ? G->comms[q]->hstage + P[q].roff : (char*)p.recv[q];
+    any_hs |= P[q].hs;
+    any_hr |= P[q].hr;
+  }
+  const size_t pe = piece_elems(p.coll, p.count, e), np = (p.count + pe - 1) / pe;
+  cudaStream_t ls = p.streams.back();
+  std::vector<cudaStream_t> others;
+  for (auto s : p.streams)
+    if (s != ls && std::find(others.begin(), others.end(), s) == others.end()) others.push_back(s);
+  HostCopy& h = G->hcopy;
+  ensure_copy(h, others.size() + 2 * np + 3);
+  size_t ei = 0;
+  for (auto s : others) {  // the launch stream joins every caller's stream
+    cuda_check(cudaEventRecord(h.ev[ei], s), "cudaEventRecord");
+    cuda_check(cudaStreamWaitEvent(ls, h.ev[ei++], 0), "cudaStreamWaitEvent");
+  }
+  cuda_check(cudaEventRecord(h.ev[ei], ls), "cudaEventRecord");
+  cuda_check(cudaStreamWaitEvent(h.h2d, h.ev[ei], 0), "cudaStreamWaitEvent");
+  cuda_check(cudaStreamWaitEvent(h.d2h, h.ev[ei++], 0), "cudaStreamWaitEvent");
+  const bool ar = p.coll == (int)Coll::AllReduce;
+  for (size_t k = 0; k < np; ++k) {
+    const size_t lo = k * pe, n = std::min(pe, p.count - lo);
+    const size_t off = ar ? lo * e : 0;
+    if (any_hs) {
+      for (int q = 0; q < N; ++q)
+        if (P[q].hs)
+          cuda_check(cudaMemcpyAsync((char*)ds[q] + off, (const char*)p.send[q] + off, ar ? n * e : P[q].sb,
+                                     cudaMemcpyHostToDevice, h.h2d), "cudaMemcpyAsync(H2D)");
+      cuda_check(cudaEventRecord(h.ev[ei], h.h2d), "cudaEventRecord");
+      cuda_check(cudaStreamWaitEvent(ls, h.ev[ei++], 0), "cudaStreamWaitEvent");
+    }
+    Pending piece = p;
+    piece.count = n;
+    piece.host = false;
+    piece.streams.assign(1, ls);
+    for (int q = 0; q < N; ++q) {
+      piece.send[q] = ds[q] + off;
+      piece.recv[q] = dr[q] + off;
+    }
+    group_launch(G, piece);
+    if (any_hr) {
+      cuda_check(cudaEventRecord(h.ev[ei], ls), "cudaEventRecord");
+      cuda_check(cudaStreamWaitEvent(h.d2h, h.ev[ei++], 0), "cudaStreamWaitEvent");
+      for (int q = 0; q < N; ++q)
+        if (P[q].hr)
+          cuda_check(cudaMemcpyAsync((char*)p.recv[q] + off, dr[q] + off, ar ? n * e : P[q].rb,
+                                     cudaMemcpyDeviceToHost, h.d2h), "cudaMemcpyAsync(D2H)");
+    }
+  }
+  if (any_hr) {
+    cuda_check(cudaEventRecord(h.ev[ei], h.d2h), "cudaEventRecord");
+    cuda_check(cudaStreamWaitEvent(ls, h.ev[ei++], 0), "cudaStreamWaitEvent");
+  }
+  cuda_check(cudaEventRecord(h.ev[ei], ls), "cudaEventRecord");  // every caller's stream after it
+  for (auto s : others) cuda_check(cudaStreamWaitEvent(s, h.ev[ei], 0), "cudaStreamWaitEvent");
+}
+
 rescclAlgo* ensure_algo(rescclComm* comm, Coll coll);
 bool try_nvls(rescclComm* comm, const AlgoShared& a, int coll, const void* send, void* recv, size_t count,
               rescclDataType_t dt, rescclRedOp_t op, cudaStream_t s);
@@ -781,12 +993,20 @@ void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t
   const bool capturing = cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone;
   if (capturing && !comm->active[coll])
     fail(rescclInvalidUsage, "load an algorithm before capturing a collective into a CUDA graph");
+  const bool host = count > 0 && (host_ptr(send) || host_ptr(recv));
+  if (capturing && host)
+    fail(rescclInvalidUsage, "host buffers cannot be captured into a CUDA graph (staged copies)");
   rescclAlgo* algo = ensure_algo(comm, (Coll)coll);
   if (capturing && (!algo->s->opt.devepoch || algo->s->opt.nvls))
     fail(rescclInvalidUsage, "this algorithm cannot be captured into a CUDA graph (devepoch=0 or nvls=1: "
                              "host-side epochs)");
   if (comm->mode != 1) {
     if (count == 0) return;
+    if (host) {
+      cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
+      host_rank(comm, algo, CallDesc{coll, count, dt, op}, send, recv, s);
+      return;
+    }
     if (algo->s->opt.nvls && try_nvls(comm, *algo->s, coll, send, recv, count, dt, op, s)) return;
     launch_rank(comm, algo, CallDesc{coll, count, dt, op}, send, recv, s);
     return;
@@ -812,12 +1032,18 @@ void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t
   p.send[comm->rank] = send;
   p.recv[comm->rank] = recv;
   p.streams.push_back(s);
+  p.host |= host;
   p.arrived++;
   while (!G->pending.empty() && G->pending.front().arrived == G->nranks) {
     Pending q = G->pending.front();
     G->pending.pop_front();
     G->base++;
-    if (q.count > 0) group_launch(G, q);
+    if (q.count > 0) {
+      if (q.host)
+        group_host_launch(G, q);
+      else
+        group_launch(G, q);
+    }
   }
 }
 
@@ -1477,11 +1703,13 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
         if (kv.second->dev_epochs) cudaFree(kv.second->dev_epochs);
       }
       for (auto e : G->events) cudaEventDestroy(e);
+      G->hcopy.release();
       cudaFreeHost(G->err_host);
-      for (auto c : G->comms)
-        if (c->scratch) cudaFree(c->scratch);
       delete G;
     }
+    // this rank's buffers (the group's other comms may already be deleted)
+    if (comm->scratch) cudaFree(comm->scratch);
+    if (comm->hstage) cudaFree(comm->hstage);
   } else {
     for (auto& a : comm->algos) {
       for (auto* e : a->dev_epochs)
@@ -1498,6 +1726,8 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
     if (comm->arena) cudaFree(comm->arena);
     if (comm->err_host) cudaFreeHost(comm->err_host);
     if (comm->scratch) cudaFree(comm->scratch);
+    if (comm->hstage) cudaFree(comm->hstage);
+    comm->hcopy.release();
   }
   delete comm;
   API_END

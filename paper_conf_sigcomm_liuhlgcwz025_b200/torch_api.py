@@ -42,7 +42,9 @@ class Communicator:
         return a
 
     def allreduce(self, send, recv, op: str = "sum", stream=None):
-        assert send.is_cuda and recv.is_cuda and send.numel() == recv.numel()
+        # device tensors, or host tensors (pinned for async copies): the library stages
+        # host buffers through device memory itself (include/resccl.h, host buffers)
+        assert send.numel() == recv.numel()
         _r.rescclAllReduce(send.data_ptr(), recv.data_ptr(), send.numel(), dtype_of(send), _r.OPS[op],
                            self.handle, _stream(stream))
 

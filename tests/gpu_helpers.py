@@ -11,11 +11,14 @@ TORCH_DT = {"int32": "int32", "float32": "float32", "float16": "float16", "bfloa
 
 
 def to_torch(x: np.ndarray, dtype: str, device="cuda:0"):
+    """device "cuda:0", "pinned" (page-locked host) or "cpu" (pageable host)."""
     import torch
     if dtype == "bfloat16":
         t = torch.from_numpy(x.view(np.int16).copy()).view(torch.bfloat16)
     else:
         t = torch.from_numpy(x.copy())
+    if device == "pinned":
+        return t.pin_memory()
     return t.to(device)
 
 
@@ -36,23 +39,30 @@ def poison(t):
 
 
 def run_virtual(R, ir_text: str, coll: str, xs, dtype: str, count: int, op: str = "sum",
-                inplace: bool = False, iters: int = 1):
+                inplace: bool = False, iters: int = 1, send_dev: str = "cuda:0", recv_dev: str = "cuda:0"):
     """Load ``ir_text`` on len(xs) virtual ranks of cuda:0, run ``iters`` times, return
-    (outputs as numpy, plan info, async error)."""
+    (outputs as numpy, plan info, async error).  send_dev / recv_dev: where the buffers
+    live ("cuda:0", "pinned" or "cpu" host memory; in-place uses send_dev for both)."""
     import torch
     n = len(xs)
     grp = R.VirtualGroup(n, 0)
     try:
         grp.load(ir_text)
         info = grp.plan_info()
-        sends = [to_torch(x, dtype) for x in xs]
+        sends = [to_torch(x, dtype, send_dev) for x in xs]
+
+        def empty(m, like):
+            if send_dev in ("pinned", "cpu") and inplace or recv_dev in ("pinned", "cpu") and not inplace:
+                t = torch.empty(m, dtype=like.dtype)
+                return t.pin_memory() if (send_dev if inplace else recv_dev) == "pinned" else t
+            return torch.empty(m, dtype=like.dtype, device="cuda:0")
         recvs = []
         for r in range(n):
             if inplace:
                 if coll == "allreduce":
                     recvs.append(sends[r])
                 elif coll == "allgather":
-                    big = torch.empty(n * count, dtype=sends[r].dtype, device="cuda:0")
+                    big = empty(n * count, sends[r])
                     poison(big)
                     big[r * count:(r + 1) * count].copy_(sends[r])
                     sends[r] = big[r * count:(r + 1) * count]
@@ -61,7 +71,7 @@ def run_virtual(R, ir_text: str, coll: str, xs, dtype: str, count: int, op: str 
                     recvs.append(sends[r][r * count:(r + 1) * count])
             else:
                 m = count * n if coll == "allgather" else count
-                t = torch.empty(m, dtype=sends[r].dtype, device="cuda:0")
+                t = empty(m, sends[r])
                 poison(t)
                 recvs.append(t)
         for _ in range(iters):
