@@ -3,6 +3,8 @@
   c3     DBT and HM 2x4 allreduce under a TB budget 1..16                   (configs[2])
   c4     synthesized allgather / reducescatter, 4..256 MiB, fanout 2/3      (configs[3])
   f2     HPDS vs round-robin sub-pipelines (Fig. 10b analogue)
+  nr     ring allreduce bf16 at 2 / 4 / 8 virtual ranks vs size (the metric's 2/4/8 axis), the
+         bench geometry with 148 // N instances per rank (every SM busy at every N)
 busBW follows nccl-tests: AR 2(N-1)/N, AG/RS (N-1)/N of algBW, S = per-rank buffer
 (AG: total output; RS: total input).  Usage: python tools/sweep.py c2 [c3 c4 f2]"""
 import json
@@ -18,7 +20,16 @@ BASE = dict(instances=18, chunkbytes=8 << 20, fifodepth=2, direct=int(os.environ
 ELT = {"bfloat16": 2, "float32": 4, "int32": 4}
 
 
-def measure(name, coll, gopts, opts, S, dtype="bfloat16", iters=10, warm=3):
+def measure(name, coll, gopts, opts, S, dtype="bfloat16", iters=10, warm=3, n=None):
+    global N
+    N0, N = N, (n or N)
+    try:
+        return _measure(name, coll, gopts, opts, S, dtype, iters, warm)
+    finally:
+        N = N0
+
+
+def _measure(name, coll, gopts, opts, S, dtype="bfloat16", iters=10, warm=3):
     text = R.rescclGenerateIr(name, coll, N, gopts)
     hdr, rest = text.split("\n", 1)
     hdr += "".join(f" {k}={v}" for k, v in opts.items())
@@ -57,7 +68,7 @@ def measure(name, coll, gopts, opts, S, dtype="bfloat16", iters=10, warm=3):
         Sb = (sn if coll != "allgather" else rn) * elt
         alg = Sb / (ms * 1e-3) / 1e9
         bus = alg * (2 * (N - 1) / N if coll == "allreduce" else (N - 1) / N)
-        return {"algo": name, "coll": coll, "gopts": gopts, "opts": opts, "dtype": dtype, "bytes": Sb,
+        return {"nranks": N, "algo": name, "coll": coll, "gopts": gopts, "opts": opts, "dtype": dtype, "bytes": Sb,
                 "us": round(ms * 1e3, 2), "algbw_gbs": round(alg, 2), "busbw_gbs": round(bus, 2),
                 "ctas_per_rank": info["ctas"], "blocks": sum(info["blocks_per_rank"]),
                 "instances": info["instances"], "linkmodel": info["linkmodel"], "fused": info["plan"]["fused"],
@@ -97,3 +108,9 @@ if "f2" in which:
         for sched in ("hpds", "rr"):
             emit(measure(name, coll, g, dict(instances=4, chunkbytes=1 << 20, fifodepth=2, sched=sched,
                                              direct=BASE["direct"]), 64 << 20))
+if "nr" in which:
+    for n in (2, 4, 8):
+        for S in [1 << k for k in range(20, 31, 2)]:
+            emit(measure("ring", "allreduce", "", dict(instances=148 // n, chunkbytes=32 << 20, fifodepth=2,
+                                                       nwarps=8, direct=BASE["direct"]), S,
+                         iters=20 if S < (64 << 20) else 10, n=n))
