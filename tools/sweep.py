@@ -111,6 +111,6 @@ if "f2" in which:
 if "nr" in which:
     for n in (2, 4, 8):
         for S in [1 << k for k in range(20, 31, 2)]:
-            emit(measure("ring", "allreduce", "", dict(instances=148 // n, chunkbytes=32 << 20, fifodepth=2,
+            emit(measure("ring", "allreduce", "", dict(instances=min(64, 148 // n), chunkbytes=32 << 20, fifodepth=2,
                                                        nwarps=8, direct=BASE["direct"]), S,
                          iters=20 if S < (64 << 20) else 10, n=n))
