@@ -142,6 +142,7 @@ struct Options {
   int l2hint = 1;
   int tma_min = 32768;   // r01 (24 KiB tiles): the TMA engine wins from 32 KiB slices (16 MiB AR +31%)
   int backoff = 1;
+  int pollacq = 0;
   int jitter = 0;
   int prefetch = 0;  // r01: L2 prefetch evicts FIFO lines and loses 10-25%
   int pool_cap = 0;  // stages of the CTA pool one lane may hold (0 = all)
@@ -196,6 +197,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "tmamin") o.tma_min = (int)to_long(v, k);
   else if (k == "direct") o.direct = (int)to_long(v, k);
   else if (k == "backoff") o.backoff = (int)to_long(v, k);
+  else if (k == "pollacq") o.pollacq = (int)to_long(v, k);
   else if (k == "jitter") o.jitter = (int)to_long(v, k);
   else if (k == "sysrank") o.sys_rank = (int)to_long(v, k);
   else if (k == "poolcap") o.pool_cap = (int)to_long(v, k);
@@ -226,7 +228,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_BULKRED", "bulkred"}, {"RESCCL_DEVEPOCH", "devepoch"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_POLL_ACQ", "pollacq"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_BULKRED", "bulkred"}, {"RESCCL_DEVEPOCH", "devepoch"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -525,6 +527,7 @@ CodegenOpts codegen_opts(const Options& o) {
   co.prefetch = o.prefetch;
   co.tma_min = o.tma_min;
   co.backoff = o.backoff;
+  co.pollacq = o.pollacq;
   co.jitter = o.jitter;
   co.pool_cap = o.pool_cap;
   co.store_lag = o.store_lag;

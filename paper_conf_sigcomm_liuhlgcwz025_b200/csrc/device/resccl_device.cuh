@@ -147,10 +147,19 @@ __device__ __forceinline__ u64 ld_relaxed(const u64* p) {
   asm volatile("ld.relaxed" RESCCL_SC ".global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+#ifndef RESCCL_POLL_ACQ
+#define RESCCL_POLL_ACQ 0
+#endif
+// RESCCL_POLL_ACQ=1: every probe is the acquire load (one L2 round trip less per handoff
+// once the value is there, an L1 invalidate per probe)
 __device__ __forceinline__ bool ready_ge(const u64* p, u64 target) {
+#if RESCCL_POLL_ACQ
+  return ld_acquire(p) >= target;
+#else
   if (ld_relaxed(p) < target) return false;
   (void)ld_acquire(p);
   return true;
+#endif
 }
 __device__ __forceinline__ u64 globaltimer() {
   u64 t;

@@ -55,6 +55,7 @@ struct CodegenOpts {
   int l2hint = 1;                // L2 evict_last on FIFO writes, evict_first on streams
   int tma_min = 32768;           // slices below this many bytes use the register path
   int backoff = 1;               // nanosleep back-off while polling flags
+  int pollacq = 0;               // poll flags with ld.acquire (no separate confirming acquire)
   int jitter = 0;                // debug fault injector: random delays around every sync
   int prefetch = 0;              // micro-batches of local operand prefetched into L2 ahead (off: r01)
   int pool_cap = 0;              // stages of the CTA pool one lane may hold (0 = all)

@@ -18,7 +18,8 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, algo, coll, count, dtype, q, opts="chunkbytes=4096 instances=2 fifodepth=2"):
+def _worker(rank, world, port, algo, coll, count, dtype, q, opts="chunkbytes=4096 instances=2 fifodepth=2",
+            where="cuda:0"):
     try:
         import sys
         root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -39,11 +40,13 @@ def _worker(rank, world, port, algo, coll, count, dtype, q, opts="chunkbytes=409
         comm.load(hdr + " " + opts + "\n" + rest)
         m = count * world if coll == "reducescatter" else count
         x = inp.rank_input(dtype, 3, rank, m)
-        s = to_torch(x, dtype)
+        s = to_torch(x, dtype, where)
         outs = []
         for it in range(2):  # two calls: monotone flags across calls
             n_out = count * world if coll == "allgather" else count
-            r = torch.empty(n_out, dtype=s.dtype, device="cuda:0")
+            r = torch.empty(n_out, dtype=s.dtype, device="cpu" if where == "pinned" else "cuda:0")
+            if where == "pinned":
+                r = r.pin_memory()
             poison(r)
             getattr(comm, coll)(s, r)
             torch.cuda.synchronize()
@@ -59,9 +62,12 @@ def _worker(rank, world, port, algo, coll, count, dtype, q, opts="chunkbytes=409
 
 
 @pytest.mark.timeout(240)
-@pytest.mark.parametrize("algo,coll,world", [("ring", "allreduce", 2), ("ring", "allgather", 2),
-                                             ("ring", "reducescatter", 2), ("dbt", "allreduce", 4)])
-def test_ipc_processes_match_oracle(algo, coll, world):
+@pytest.mark.parametrize("algo,coll,world,where", [("ring", "allreduce", 2, "cuda:0"), ("ring", "allgather", 2, "cuda:0"),
+                                                   ("ring", "reducescatter", 2, "cuda:0"), ("dbt", "allreduce", 4, "cuda:0"),
+                                                   ("ring", "allreduce", 2, "pinned"), ("ring", "allgather", 2, "pinned"),
+                                                   ("ring", "reducescatter", 2, "pinned")])
+def test_ipc_processes_match_oracle(algo, coll, world, where):
+    """where = "pinned": host send/receive buffers, staged by the library (host_rank)."""
     import torch.multiprocessing as mp
     import resccl_inputs as inp
     from oracle import ir as oir, lower, replay
@@ -71,7 +77,8 @@ def test_ipc_processes_match_oracle(algo, coll, world):
     port = _free_port()
     env_old = os.environ.get("RESCCL_TIMEOUT_MS")
     os.environ["RESCCL_TIMEOUT_MS"] = "60000"
-    procs = [ctx.Process(target=_worker, args=(r, world, port, algo, coll, count, dtype, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, algo, coll, count, dtype, q),
+                         kwargs={"where": where}) for r in range(world)]
     for p in procs:
         p.start()
     res = {}
