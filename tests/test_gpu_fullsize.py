@@ -28,7 +28,13 @@ def _positions(geo, c, rng, n_rand=3000):
 
 @pytest.mark.timeout(600)
 @pytest.mark.parametrize("algo,n,size_mb,dtype,opts", [
-    ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=4 << 20, fifodepth=2)),   # bench.py default
+    # bench.py's N=1 launch configuration (headline line, then its in-place line)
+    ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=1)),
+    ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=1,
+                                      _inplace=True)),
+    # the C2 sweep's largest size, same geometry
+    ("ring", 8, 1024, "bfloat16", dict(instances=18, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=1)),
+    ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=4 << 20, fifodepth=2)),
     ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=4 << 20, fifodepth=2, direct=1)),
     ("ring", 8, 64, "float32", dict(instances=16, chunkbytes=2 << 20, fifodepth=2)),
     ("hm", 8, 64, "bfloat16", dict(instances=4, chunkbytes=1 << 20, fifodepth=2)),
@@ -39,6 +45,8 @@ def test_fullsize_sampled(algo, n, size_mb, dtype, opts):
     import paper_conf_sigcomm_liuhlgcwz025_b200 as R
     elt = {"bfloat16": 2, "float16": 2, "float32": 4}[dtype]
     count = size_mb * (1 << 20) // elt
+    opts = dict(opts)
+    inplace = opts.pop("_inplace", False)
     g = oir.generate(algo, "allreduce", n, **({"g": 4} if algo == "hm" else {}))
     for k, v in opts.items():
         g.extra[k] = str(v)
@@ -46,12 +54,17 @@ def test_fullsize_sampled(algo, n, size_mb, dtype, opts):
     try:
         grp.load(g.to_text())
         sends = [inp.rank_input_torch(dtype, 11, r, count) for r in range(n)]
-        recvs = [torch.empty_like(s) for s in sends]
-        for _ in range(2):
-            for t in recvs:
-                t.fill_(float("nan"))
-            grp.allreduce(sends, recvs)
+        if inplace:  # one call: the result replaces the input
+            grp.allreduce(sends, sends)
             torch.cuda.synchronize()
+            recvs = sends
+        else:
+            recvs = [torch.empty_like(s) for s in sends]
+            for _ in range(2):
+                for t in recvs:
+                    t.fill_(float("nan"))
+                grp.allreduce(sends, recvs)
+                torch.cuda.synchronize()
         assert grp.async_error() == 0
         geo = replay.Geometry("allreduce", n, count, elt, opts["chunkbytes"], opts["instances"])
         rng = np.random.default_rng(0)
