@@ -373,7 +373,8 @@ def main():
         e2e_bus = S / (ems * 1e-3) / 1e9 * 2 * (n - 1) / n
         e2e = {"value": round(e2e_bus, 3), "unit": "GB/s", "h2d_bytes_per_step": S * len(my_ranks),
                "d2h_bytes_per_step": S * len(my_ranks), "ms_per_step": round(ems, 3),
-               "path": "C-ABI collective on pinned host buffers (library-staged, piecewise H2D/AR/D2H overlap)"}
+               "path": "C-ABI collective on pinned host buffers (library-staged, piecewise H2D/AR/D2H overlap)",
+               "piece_bytes": int(os.environ.get("RESCCL_HOST_PIECE", 32 << 20))}
         if dmax is not None:
             e2e["max_abs_diff_vs_device_result"] = dmax
             e2e["within_tolerance"] = bool(dmax <= 2e-2 * n) if tdt.is_floating_point else bool(dmax == 0)

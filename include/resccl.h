@@ -28,9 +28,12 @@
  *    stages it through device memory the communicator owns (grown on demand, freed
  *    by rescclCommDestroy): uploads on an internal copy stream, the collective on
  *    `stream`, downloads on a second copy stream, and `stream` waits for the last
- *    download, so the result is in recvbuf once `stream` completes.  AllReduce is
- *    cut into pieces of RESCCL_HOST_PIECE bytes (default 32 MiB) whose upload,
- *    collective and download overlap.  The host in-place rules are the device ones.
+ *    download, so the result is in recvbuf once `stream` completes.  A call is cut
+ *    into pieces of RESCCL_HOST_PIECE bytes per rank (default 32 MiB) whose upload,
+ *    collective and download overlap; each piece is a collective of its own over the
+ *    piece's columns (its own chunk layout, so fp sums may round differently from one
+ *    unpieced call).  An AllGather with a device recvbuf or a ReduceScatter with a
+ *    device sendbuf runs as one piece.  The host in-place rules are the device ones.
  *    Host-buffer calls refuse CUDA-graph capture (InvalidUsage).  Staged calls of a
  *    direct=1 algorithm across processes run its staged twin (the stage is not a
  *    registered window).

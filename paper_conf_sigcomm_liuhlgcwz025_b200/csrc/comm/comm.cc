@@ -787,9 +787,10 @@ void group_launch(Group* G, Pending& p) {
 // ------------------------------------------------------------ host-buffer collectives
 // A send or receive buffer in host memory (pinned, or pageable at pageable-copy speed) is
 // staged through device memory the communicator owns: upload on a copy stream, the
-// collective on the caller's stream, download on a second copy stream.  AllReduce is cut
-// into pieces of RESCCL_HOST_PIECE bytes (default 32 MiB) so that piece k's collective
-// and piece k-1's download overlap piece k+1's upload (PCIe is full duplex).  The
+// collective on the caller's stream, download on a second copy stream.  A call is cut
+// into pieces of RESCCL_HOST_PIECE bytes per rank (default 32 MiB; layout at Staging) so
+// that piece k's collective and piece k-1's download overlap piece k+1's upload (PCIe is
+// full duplex).  The
 // caller's stream waits for the last download: stream semantics are the device path's.
 
 bool host_ptr(const void* p) {
@@ -833,50 +834,82 @@ void ensure_copy(HostCopy& h, size_t nev) {
   }
 }
 
-// One rank's staging: device offsets of the send / receive regions in its stage (-1 =
-// the caller's device buffer).  Host in-place calls (NCCL's rules: AR send == recv, AG
-// send == recv + rank*count, RS recv == send + rank*count) stage one region.
-struct StagePlan {
-  size_t sb = 0, rb = 0, need = 0;
-  long long soff = -1, roff = -1;
-  bool hs = false, hr = false;
+// One rank's staging.  A call is cut into pieces [lo, lo+m) of the per-rank count: AR
+// pieces are contiguous; an AllGather piece's output and a ReduceScatter piece's input are
+// N rows of m elements, so their stage regions are piece-major (piece k's N*m block at
+// N*lo) and the strided host side moves with 2D copies.  A device-side AG output or RS
+// input cannot be piece-major: such calls run as one piece.  Host in-place calls (NCCL's
+// rules: AR send == recv, AG send == recv + rank*count, RS recv == send + rank*count)
+// stage one region.
+struct Staging {
+  int coll = 0, rank = 0, N = 1;
+  size_t count = 0, e = 0, sb = 0, rb = 0, need = 0;
+  long long soff = -1, roff = -1;  // stage offsets of the send / receive regions (-1: caller's buffer)
+  bool hs = false, hr = false, inplace = false, pieces = false;
+  const char* send = nullptr;
+  char* recv = nullptr;
+  char* stage = nullptr;
+
+  void plan(int coll_, int rank_, int N_, const void* send_, void* recv_, size_t count_, size_t e_) {
+    coll = coll_, rank = rank_, N = N_, count = count_, e = e_;
+    send = (const char*)send_, recv = (char*)recv_;
+    sb = count * e * (coll == (int)Coll::ReduceScatter ? N : 1);
+    rb = count * e * (coll == (int)Coll::AllGather ? N : 1);
+    hs = host_ptr(send);
+    hr = host_ptr(recv);
+    const size_t blk = (size_t)rank * count * e;
+    if (hs && hr && coll == (int)Coll::AllReduce && send == recv) {
+      inplace = true, need = rb, soff = roff = 0;
+    } else if (hs && hr && coll == (int)Coll::AllGather && send == recv + blk) {
+      inplace = true, need = rb, roff = 0, soff = (long long)blk;
+    } else if (hs && hr && coll == (int)Coll::ReduceScatter && recv == send + blk) {
+      inplace = true, need = sb, soff = 0, roff = (long long)blk;
+    } else {
+      if (hs) soff = 0, need += sb;
+      if (hr) roff = (long long)need, need += rb;
+    }
+    pieces = coll == (int)Coll::AllReduce || (coll == (int)Coll::AllGather ? hr : hs);
+  }
+  // device buffers of piece [lo, lo+m)
+  const char* dsend(size_t lo, size_t m) const {
+    if (coll == (int)Coll::AllGather && inplace) return drecv(lo, m) + (size_t)rank * m * e;
+    const char* base = soff >= 0 ? stage + soff : send;
+    return base + (coll == (int)Coll::ReduceScatter ? (size_t)N : 1) * lo * e;
+  }
+  char* drecv(size_t lo, size_t m) const {
+    if (coll == (int)Coll::ReduceScatter && inplace) return (char*)dsend(lo, m) + (size_t)rank * m * e;
+    char* base = roff >= 0 ? stage + roff : recv;
+    return base + (coll == (int)Coll::AllGather ? (size_t)N : 1) * lo * e;
+  }
+  void upload(size_t lo, size_t m, cudaStream_t st) const {
+    char* d = (char*)dsend(lo, m);
+    if (coll == (int)Coll::ReduceScatter)  // N rows: host pitch count, stage pitch m
+      cuda_check(cudaMemcpy2DAsync(d, m * e, send + lo * e, count * e, m * e, N, cudaMemcpyHostToDevice, st),
+                 "cudaMemcpy2DAsync(H2D)");
+    else
+      cuda_check(cudaMemcpyAsync(d, send + lo * e, m * e, cudaMemcpyHostToDevice, st), "cudaMemcpyAsync(H2D)");
+  }
+  void download(size_t lo, size_t m, cudaStream_t st) const {
+    const char* d = drecv(lo, m);
+    if (coll == (int)Coll::AllGather)
+      cuda_check(cudaMemcpy2DAsync(recv + lo * e, count * e, d, m * e, m * e, N, cudaMemcpyDeviceToHost, st),
+                 "cudaMemcpy2DAsync(D2H)");
+    else
+      cuda_check(cudaMemcpyAsync(recv + lo * e, d, m * e, cudaMemcpyDeviceToHost, st), "cudaMemcpyAsync(D2H)");
+  }
 };
 
-StagePlan stage_plan(int coll, int rank, int nranks, const void* send, void* recv, size_t count, size_t e) {
-  StagePlan P;
-  P.sb = count * e * (coll == (int)Coll::ReduceScatter ? nranks : 1);
-  P.rb = count * e * (coll == (int)Coll::AllGather ? nranks : 1);
-  P.hs = host_ptr(send);
-  P.hr = host_ptr(recv);
-  const char* sp = (const char*)send;
-  const char* rp = (const char*)recv;
-  const size_t blk = (size_t)rank * count * e;
-  if (P.hs && P.hr && coll == (int)Coll::AllReduce && sp == rp) {
-    P.need = P.rb, P.soff = P.roff = 0;
-  } else if (P.hs && P.hr && coll == (int)Coll::AllGather && sp == rp + blk) {
-    P.need = P.rb, P.roff = 0, P.soff = (long long)blk;
-  } else if (P.hs && P.hr && coll == (int)Coll::ReduceScatter && rp == sp + blk) {
-    P.need = P.sb, P.soff = 0, P.roff = (long long)blk;
-  } else {
-    if (P.hs) P.soff = 0, P.need += P.sb;
-    if (P.hr) P.roff = (long long)P.need, P.need += P.rb;
-  }
-  return P;
-}
-
-size_t piece_elems(int coll, size_t count, size_t e) {
-  return coll == (int)Coll::AllReduce ? std::min(count, std::max<size_t>(1, host_piece_bytes() / e)) : count;
-}
+size_t piece_elems(size_t count, size_t e) { return std::min(count, std::max<size_t>(1, host_piece_bytes() / e)); }
 
 // multi-process / multi-device rank
 void host_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const void* send, void* recv,
                cudaStream_t s) {
   const size_t e = elt_size(c.dt);
-  const StagePlan P = stage_plan(c.coll, comm->rank, comm->nranks, send, recv, c.count, e);
+  Staging P;
+  P.plan(c.coll, comm->rank, comm->nranks, send, recv, c.count, e);
   ensure_hstage(comm, P.need);
-  const char* ds = P.soff >= 0 ? comm->hstage + P.soff : (const char*)send;
-  char* dr = P.roff >= 0 ? comm->hstage + P.roff : (char*)recv;
-  const size_t pe = piece_elems(c.coll, c.count, e), np = (c.count + pe - 1) / pe;
+  P.stage = comm->hstage;
+  const size_t pe = P.pieces ? piece_elems(c.count, e) : c.count, np = (c.count + pe - 1) / pe;
   HostCopy& h = comm->hcopy;
   ensure_copy(h, 2 * np + 2);
   size_t ei = 0;
@@ -884,20 +917,17 @@ void host_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const void
   cuda_check(cudaStreamWaitEvent(h.h2d, h.ev[ei], 0), "cudaStreamWaitEvent");
   cuda_check(cudaStreamWaitEvent(h.d2h, h.ev[ei++], 0), "cudaStreamWaitEvent");
   for (size_t k = 0; k < np; ++k) {
-    const size_t lo = k * pe, n = std::min(pe, c.count - lo);
-    const size_t off = c.coll == (int)Coll::AllReduce ? lo * e : 0;
+    const size_t lo = k * pe, m = std::min(pe, c.count - lo);
     if (P.hs) {
-      cuda_check(cudaMemcpyAsync((char*)ds + off, (const char*)send + off, c.coll == (int)Coll::AllReduce ? n * e : P.sb,
-                                 cudaMemcpyHostToDevice, h.h2d), "cudaMemcpyAsync(H2D)");
+      P.upload(lo, m, h.h2d);
       cuda_check(cudaEventRecord(h.ev[ei], h.h2d), "cudaEventRecord");
       cuda_check(cudaStreamWaitEvent(s, h.ev[ei++], 0), "cudaStreamWaitEvent");
     }
-    launch_rank(comm, algo, CallDesc{c.coll, n, c.dt, c.op}, ds + off, dr + off, s);
+    launch_rank(comm, algo, CallDesc{c.coll, m, c.dt, c.op}, P.dsend(lo, m), P.drecv(lo, m), s);
     if (P.hr) {
       cuda_check(cudaEventRecord(h.ev[ei], s), "cudaEventRecord");
       cuda_check(cudaStreamWaitEvent(h.d2h, h.ev[ei++], 0), "cudaStreamWaitEvent");
-      cuda_check(cudaMemcpyAsync((char*)recv + off, dr + off, c.coll == (int)Coll::AllReduce ? n * e : P.rb,
-                                 cudaMemcpyDeviceToHost, h.d2h), "cudaMemcpyAsync(D2H)");
+      P.download(lo, m, h.d2h);
     }
   }
   if (P.hr) {
@@ -911,19 +941,17 @@ void group_host_launch(Group* G, Pending& p) {
   const int N = G->nranks;
   const size_t e = elt_size((rescclDataType_t)p.dtype);
   cuda_check(cudaSetDevice(G->dev), "cudaSetDevice");
-  std::vector<StagePlan> P(N);
-  std::vector<const char*> ds(N);
-  std::vector<char*> dr(N);
-  bool any_hs = false, any_hr = false;
+  std::vector<Staging> P(N);
+  bool any_hs = false, any_hr = false, pieces = true;
   for (int q = 0; q < N; ++q) {
-    P[q] = stage_plan(p.coll, q, N, p.send[q], p.recv[q], p.count, e);
+    P[q].plan(p.coll, q, N, p.send[q], p.recv[q], p.count, e);
     ensure_hstage(G->comms[q], P[q].need);
-    ds[q] = P[q].soff >= 0 ? G->comms[q]->hstage + P[q].soff : (const char*)p.send[q];
-    dr[q] = P[q].roff >= 0 ? G->comms[q]->hstage + P[q].roff : (char*)p.recv[q];
+    P[q].stage = G->comms[q]->hstage;
     any_hs |= P[q].hs;
     any_hr |= P[q].hr;
+    pieces &= P[q].pieces;
   }
-  const size_t pe = piece_elems(p.coll, p.count, e), np = (p.count + pe - 1) / pe;
+  const size_t pe = pieces ? piece_elems(p.count, e) : p.count, np = (p.count + pe - 1) / pe;
   cudaStream_t ls = p.streams.back();
   std::vector<cudaStream_t> others;
   for (auto s : p.streams)
@@ -938,34 +966,28 @@ void group_host_launch(Group* G, Pending& p) {
   cuda_check(cudaEventRecord(h.ev[ei], ls), "cudaEventRecord");
   cuda_check(cudaStreamWaitEvent(h.h2d, h.ev[ei], 0), "cudaStreamWaitEvent");
   cuda_check(cudaStreamWaitEvent(h.d2h, h.ev[ei++], 0), "cudaStreamWaitEvent");
-  const bool ar = p.coll == (int)Coll::AllReduce;
   for (size_t k = 0; k < np; ++k) {
-    const size_t lo = k * pe, n = std::min(pe, p.count - lo);
-    const size_t off = ar ? lo * e : 0;
+    const size_t lo = k * pe, m = std::min(pe, p.count - lo);
     if (any_hs) {
       for (int q = 0; q < N; ++q)
-        if (P[q].hs)
-          cuda_check(cudaMemcpyAsync((char*)ds[q] + off, (const char*)p.send[q] + off, ar ? n * e : P[q].sb,
-                                     cudaMemcpyHostToDevice, h.h2d), "cudaMemcpyAsync(H2D)");
+        if (P[q].hs) P[q].upload(lo, m, h.h2d);
       cuda_check(cudaEventRecord(h.ev[ei], h.h2d), "cudaEventRecord");
       cuda_check(cudaStreamWaitEvent(ls, h.ev[ei++], 0), "cudaStreamWaitEvent");
     }
     Pending piece = p;
-    piece.count = n;
+    piece.count = m;
     piece.host = false;
     piece.streams.assign(1, ls);
     for (int q = 0; q < N; ++q) {
-      piece.send[q] = ds[q] + off;
-      piece.recv[q] = dr[q] + off;
+      piece.send[q] = P[q].dsend(lo, m);
+      piece.recv[q] = P[q].drecv(lo, m);
     }
     group_launch(G, piece);
     if (any_hr) {
       cuda_check(cudaEventRecord(h.ev[ei], ls), "cudaEventRecord");
       cuda_check(cudaStreamWaitEvent(h.d2h, h.ev[ei++], 0), "cudaStreamWaitEvent");
       for (int q = 0; q < N; ++q)
-        if (P[q].hr)
-          cuda_check(cudaMemcpyAsync((char*)p.recv[q] + off, dr[q] + off, ar ? n * e : P[q].rb,
-                                     cudaMemcpyDeviceToHost, h.d2h), "cudaMemcpyAsync(D2H)");
+        if (P[q].hr) P[q].download(lo, m, h.d2h);
     }
   }
   if (any_hr) {

@@ -60,24 +60,48 @@ def test_host_buffers_bit_exact(coll, where, inplace):
     _same(outs, oracle_expect(g, xs, dtype, count, chunk_bytes=4096, instances=2))
 
 
-@pytest.mark.parametrize("dtype", ["float32", "bfloat16", "int32"])
-def test_host_allreduce_in_pieces(dtype, monkeypatch):
-    """RESCCL_HOST_PIECE = 8 KiB: the AllReduce runs as 4 pieces (the last ragged), each
-    bit-exact to the oracle's replay of that piece; int32 also equals the definition."""
-    n, count = 8, 3 * 2048 + 513 if dtype != "bfloat16" else 3 * 4096 + 513
+def _piece_expect(g, coll, xs, dtype, count, pe, n, **kw):
+    """Concatenation of the oracle's replays of the pieces [lo, lo+m) of the per-rank
+    count: AR / AG inputs are column slices of each rank's buffer, RS inputs the column
+    slice of each of its N rows; AG outputs interleave back into N rows."""
+    cols = []
+    for lo in range(0, count, pe):
+        m = min(pe, count - lo)
+        if coll == "reducescatter":
+            ins = [np.concatenate([x[q * count + lo:q * count + lo + m] for q in range(n)]) for x in xs]
+        else:
+            ins = [x[lo:lo + m] for x in xs]
+        cols.append((m, oracle_expect(g, ins, dtype, m, **kw)))
+    if coll != "allgather":
+        return [np.concatenate([c[r] for _, c in cols]) for r in range(n)]
+    return [np.concatenate([np.concatenate([c[r][q * m:(q + 1) * m] for m, c in cols]) for q in range(n)])
+            for r in range(n)]
+
+
+@pytest.mark.parametrize("coll,dtype", [("allreduce", "float32"), ("allreduce", "bfloat16"), ("allreduce", "int32"),
+                                        ("allgather", "bfloat16"), ("reducescatter", "float32"),
+                                        ("reducescatter", "bfloat16")])
+@pytest.mark.parametrize("where", [("pinned", "pinned"), ("pinned", "cuda:0"), ("cuda:0", "pinned")])
+def test_host_collectives_in_pieces(coll, dtype, where, monkeypatch):
+    """RESCCL_HOST_PIECE = 8 KiB: the call runs as 4 pieces (the last ragged), each
+    bit-exact to the oracle's replay of that piece (AG outputs and RS inputs move as N
+    strided rows).  A device-side AG output / RS input runs as one piece.  int32 AR also
+    equals the definition."""
+    send_dev, recv_dev = where
+    n = 8
+    elt = 2 if dtype == "bfloat16" else 4
+    pe = 8192 // elt
+    count = 3 * pe + 513
     monkeypatch.setenv("RESCCL_HOST_PIECE", str(8192))
-    pe = 8192 // (2 if dtype == "bfloat16" else 4)
-    g, text = _text("allreduce", n, chunkbytes=2048, instances=2)
-    xs = _inputs("allreduce", dtype, n, count, seed=5)
-    for inplace in (False, True):
-        outs, _, err = run_virtual(R, text, "allreduce", xs, dtype, count, inplace=inplace, send_dev="pinned",
-                                   recv_dev="pinned")
+    g, text = _text(coll, n, chunkbytes=2048, instances=2)
+    xs = _inputs(coll, dtype, n, count, seed=5)
+    one_piece = (coll == "allgather" and recv_dev == "cuda:0") or (coll == "reducescatter" and send_dev == "cuda:0")
+    kw = dict(chunk_bytes=2048, instances=2)
+    exp = oracle_expect(g, xs, dtype, count, **kw) if one_piece else _piece_expect(g, coll, xs, dtype, count, pe, n, **kw)
+    for inplace in ((False, True) if send_dev == recv_dev else (False,)):
+        outs, _, err = run_virtual(R, text, coll, xs, dtype, count, inplace=inplace, send_dev=send_dev,
+                                   recv_dev=recv_dev)
         assert err == 0
-        parts = []
-        for lo in range(0, count, pe):
-            m = min(pe, count - lo)
-            parts.append(oracle_expect(g, [x[lo:lo + m] for x in xs], dtype, m, chunk_bytes=2048, instances=2))
-        exp = [np.concatenate([p[r] for p in parts]) for r in range(n)]
         _same(outs, exp)
         if dtype == "int32":
             _same(outs, definition.allreduce(xs, dtype))
