@@ -246,13 +246,15 @@ def main():
     # at N=1 every virtual rank's buffers share one address space, under torchrun (N>1) the
     # send and receive buffers sit in a registered symmetric window.  The lane engine's
     # cost is per TMA tile, so tiles are 24 KiB (2 stages per lane, one CTA per SM):
-    #   N=1: 18 instances x 8 virtual ranks = 144 CTAs of 256 threads, 32 MiB transfer
-    #        chunks (one micro-batch per 32 MiB algorithm chunk);
+    #   N=1: 14 instances x 8 virtual ranks = 112 CTAs of 256 threads (the smallest count
+    #        within noise of the best busBW, profiles/r01_ctas_nranks.jsonl: ResCCL's
+    #        point is fewer TBs), 32 MiB transfer chunks (one micro-batch
+    #        per 32 MiB algorithm chunk);
     #   N>1: 24 CTAs of 512 threads per rank (the best per-SM geometry: 87-91 GB/s of HBM
     #        per SM at <= 32 CTAs), 8 MiB chunks.
     direct = 1 if args.direct < 0 else args.direct
     tuned = direct and not args.instances and not args.nwarps
-    inst = args.instances or ((18 if not multi else 24) if tuned else 18)
+    inst = args.instances or ((14 if not multi else 24) if tuned else 18)
     opts = {"instances": inst,
             "chunkbytes": args.chunk_bytes or ((32 << 20) if (tuned and not multi) else (8 << 20) if direct
                                                else (4 << 20)),

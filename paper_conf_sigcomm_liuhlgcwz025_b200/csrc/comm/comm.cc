@@ -2050,7 +2050,8 @@ rescclResult_t rescclProfilePlanner(const char* program, const char* opts, int v
       << ",\"subpipelines\":" << pr.size() << ",\"max_ctas_per_rank\":" << max_cta
       << ",\"parse_ms\":" << ms(t0, t1) << ",\"analysis_ms\":" << ms(t1, t2) << ",\"schedule_ms\":" << ms(t2, t3)
       << ",\"lower_ms\":" << ms(t3, t4) << ",\"verify_ms\":" << ms(t4, t5)
-      << ",\"deadlock_free\":" << (ok ? "true" : "false") << ",\"rank0_src_bytes\":" << src.size() << "}";
+      << ",\"deadlock_free\":" << (verify ? (ok ? "true" : "false") : "null")  // null: not checked
+      << ",\"rank0_src_bytes\":" << src.size() << "}";
   write_out(out.str(), json, len);
   API_END
 }

@@ -89,11 +89,16 @@ class Communicator:
 
 class VirtualGroup:
     """N virtual ranks on one GPU; every collective is issued for all ranks and runs
-    as one kernel (see resccl.h, "Execution modes")."""
+    as one kernel (see resccl.h, "Execution modes").  With ``devices`` (distinct GPUs,
+    one rank each) the same object drives the single-process multi-device mode: one
+    kernel per rank over peer memory (cudaDeviceEnablePeerAccess, NVLink)."""
 
-    def __init__(self, nranks: int, device: int = 0):
-        self.comms = [Communicator(h) for h in _r.rescclCommInitAll([device] * nranks)]
+    def __init__(self, nranks: int, device: int = 0, devices: Optional[Sequence[int]] = None):
+        devs = list(devices) if devices is not None else [device] * nranks
+        assert len(devs) == nranks
+        self.comms = [Communicator(h) for h in _r.rescclCommInitAll(devs)]
         self.nranks = nranks
+        self.devices = devs
 
     def load(self, ir_text: str) -> List[int]:
         return [c.load(ir_text) for c in self.comms]

@@ -1,5 +1,5 @@
 """f4: PyTorch DDP with its gradient-bucket AllReduce replaced by ResCCL (comm hook).
-Two processes on cuda:0 (CUDA IPC); the resulting gradients equal the manual average
+Two processes on cuda:(rank % device_count) (CUDA IPC; NVLink on a multi-GPU box); the resulting gradients equal the manual average
 of both ranks' local gradients."""
 import os
 import socket
@@ -30,16 +30,17 @@ def _worker(rank, world, port, q):
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
         dist.init_process_group("gloo", rank=rank, world_size=world)
-        torch.cuda.set_device(0)
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
         torch.manual_seed(0)
         model = torch.nn.Sequential(torch.nn.Linear(256, 512), torch.nn.GELU(), torch.nn.Linear(512, 64)).cuda()
         ref = [p.detach().clone() for p in model.parameters()]
-        comm = R.init_process_group_comm(rank, world, 0)
-        ddp = torch.nn.parallel.DistributedDataParallel(model, device_ids=[0], bucket_cap_mb=1)
+        comm = R.init_process_group_comm(rank, world, dev)
+        ddp = torch.nn.parallel.DistributedDataParallel(model, device_ids=[dev], bucket_cap_mb=1)
         state = ResCCLHookState(comm)
         ddp.register_comm_hook(state, resccl_allreduce_hook)
         torch.manual_seed(100 + rank)
-        x = torch.randn(32, 256, device="cuda:0")
+        x = torch.randn(32, 256, device=f"cuda:{dev}")
         loss = ddp(x).square().mean()
         loss.backward()
         torch.cuda.synchronize()

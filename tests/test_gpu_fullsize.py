@@ -1,7 +1,13 @@
-"""Parity at BASELINE's full sizes in bench.py's launch configuration, on sampled
-outputs: every rank's result at sampled positions (random + chunk / micro-batch /
-instance-slice boundaries) equals the oracle's step-order dataflow evaluation of the
-same IR (same association order, R8) on the same seeded inputs."""
+"""Parity at BASELINE's full sizes in bench.py's launch configuration.
+
+``test_fullsize_elementwise``: bench.py's N=1 workload (8 x 256 MiB bf16 ring AllReduce,
+its exact launch geometry, out of place and in place) compared on EVERY element of every
+rank's result with the oracle's step-order dataflow evaluation of the same IR
+(``replay.dataflow_values``, pinned to the blocking replay in
+``tests/test_oracle_pins_r2.py``), one algorithm chunk at a time on the host.
+
+The other tests compare sampled outputs (random + chunk / micro-batch / instance-slice
+boundaries) at sizes where a full host evaluation would take minutes."""
 import numpy as np
 import pytest
 
@@ -26,14 +32,52 @@ def _positions(geo, c, rng, n_rand=3000):
     return np.array(sorted(pts), dtype=np.int64)
 
 
+# bench.py's N=1 launch configuration (bench.py: instances 14 x 8 ranks = 112 CTAs)
+BENCH_OPTS = dict(instances=14, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=1, tmastages=2, tmatile=24576)
+
+
+@pytest.mark.timeout(900)
+@pytest.mark.parametrize("inplace", [False, True])
+def test_fullsize_elementwise(inplace):
+    import torch
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    n, dtype, seed = 8, "bfloat16", 11
+    count = 256 * (1 << 20) // 2
+    g = oir.generate("ring", "allreduce", n)
+    for k, v in BENCH_OPTS.items():
+        g.extra[k] = str(v)
+    grp = R.VirtualGroup(n, 0)
+    try:
+        grp.load(g.to_text())
+        sends = [inp.rank_input_torch(dtype, seed, r, count) for r in range(n)]
+        recvs = sends if inplace else [torch.full_like(s, float("nan")) for s in sends]
+        grp.allreduce(sends, recvs)
+        torch.cuda.synchronize()
+        assert grp.async_error() == 0
+        geo = replay.Geometry("allreduce", n, count, 2, BENCH_OPTS["chunkbytes"], BENCH_OPTS["instances"])
+        checked = 0
+        for c in range(n):
+            L = geo.chunk_len[c]
+            if L == 0:
+                continue
+            # chunk c of every rank's input, straight from the shared recipe (numpy)
+            ci = [[inp.rank_input(dtype, seed, r, L, offset=c * geo.C) if cc == c else np.zeros(0, np.uint16)
+                   for cc in range(n)] for r in range(n)]
+            exp = replay.dataflow_values(g, ci, dtype)
+            for r in range(n):
+                got = recvs[r][c * geo.C:c * geo.C + L].cpu().view(torch.int16).numpy().view(np.uint16)
+                bad = np.flatnonzero(got != exp[r][c])
+                assert bad.size == 0, (r, c, bad[:5], got[bad[:5]], exp[r][c][bad[:5]])
+                checked += L
+        assert checked == n * count  # every element of every rank
+    finally:
+        grp.destroy()
+
+
 @pytest.mark.timeout(600)
 @pytest.mark.parametrize("algo,n,size_mb,dtype,opts", [
-    # bench.py's N=1 launch configuration (headline line, then its in-place line)
-    ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=1)),
-    ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=1,
-                                      _inplace=True)),
-    # the C2 sweep's largest size, same geometry
-    ("ring", 8, 1024, "bfloat16", dict(instances=18, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=1)),
+    # the C2 sweep's largest size in the bench geometry
+    ("ring", 8, 1024, "bfloat16", BENCH_OPTS),
     ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=4 << 20, fifodepth=2)),
     ("ring", 8, 256, "bfloat16", dict(instances=18, chunkbytes=4 << 20, fifodepth=2, direct=1)),
     ("ring", 8, 64, "float32", dict(instances=16, chunkbytes=2 << 20, fifodepth=2)),

@@ -1,6 +1,7 @@
 """Multi-process path (one process per rank, CUDA-IPC-mapped peer arenas, .sys-scope
-flags) exercised with every process on cuda:0 -- the gpurun boxes have one GPU; CUDA
-IPC works between processes of one device.  Results are compared with the oracle."""
+flags).  Rank r runs on cuda:(r % device_count): on a one-GPU box every process shares
+cuda:0 (CUDA IPC works between processes of one device); on a multi-GPU box the same
+tests cross NVLink.  Results are compared with the oracle."""
 import os
 import socket
 
@@ -33,18 +34,19 @@ def _worker(rank, world, port, algo, coll, count, dtype, q, opts="chunkbytes=409
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
         dist.init_process_group("gloo", rank=rank, world_size=world)
-        torch.cuda.set_device(0)
-        comm = R.init_process_group_comm(rank, world, 0)
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
+        comm = R.init_process_group_comm(rank, world, dev)
         text = R.rescclGenerateIr(algo, coll, world)
         hdr, rest = text.split("\n", 1)
         comm.load(hdr + " " + opts + "\n" + rest)
         m = count * world if coll == "reducescatter" else count
         x = inp.rank_input(dtype, 3, rank, m)
-        s = to_torch(x, dtype, where)
+        s = to_torch(x, dtype, f"cuda:{dev}" if where.startswith("cuda") else where)
         outs = []
         for it in range(2):  # two calls: monotone flags across calls
             n_out = count * world if coll == "allgather" else count
-            r = torch.empty(n_out, dtype=s.dtype, device="cpu" if where == "pinned" else "cuda:0")
+            r = torch.empty(n_out, dtype=s.dtype, device="cpu" if where == "pinned" else f"cuda:{dev}")
             if where == "pinned":
                 r = r.pin_memory()
             poison(r)
@@ -152,23 +154,24 @@ def _window_worker(rank, world, port, algo, coll, count, dtype, q, opts):
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
         dist.init_process_group("gloo", rank=rank, world_size=world)
-        torch.cuda.set_device(0)
-        comm = R.init_process_group_comm(rank, world, 0)
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
+        comm = R.init_process_group_comm(rank, world, dev)
         text = R.rescclGenerateIr(algo, coll, world)
         hdr, rest = text.split("\n", 1)
         comm.load(hdr + " " + opts + "\n" + rest)
         m = count * world if coll == "reducescatter" else count
         n_out = count * world if coll == "allgather" else count
-        x = to_torch(inp.rank_input(dtype, 3, rank, m), dtype)
+        x = to_torch(inp.rank_input(dtype, 3, rank, m), dtype, f"cuda:{dev}")
         # one window holding send and receive buffers at symmetric offsets
-        win = torch.empty(m + n_out + 64, dtype=x.dtype, device="cuda:0")
+        win = torch.empty(m + n_out + 64, dtype=x.dtype, device=f"cuda:{dev}")
         comm.register(win)
         s_reg, r_reg = win[:m], win[m + 64:m + 64 + n_out]
         s_reg.copy_(x)
         outs = []
         for it, reg in enumerate([True, False, True, True]):
             s = s_reg if reg else x
-            r = r_reg if reg else torch.empty(n_out, dtype=x.dtype, device="cuda:0")
+            r = r_reg if reg else torch.empty(n_out, dtype=x.dtype, device=f"cuda:{dev}")
             poison(r)
             torch.cuda.synchronize()
             dist.barrier()
@@ -244,17 +247,18 @@ def _graph_worker(rank, world, port, count, q):
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
         dist.init_process_group("gloo", rank=rank, world_size=world)
-        torch.cuda.set_device(0)
-        comm = R.init_process_group_comm(rank, world, 0)
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
+        comm = R.init_process_group_comm(rank, world, dev)
         text = R.rescclGenerateIr("ring", "allreduce", world)
         hdr, rest = text.split("\n", 1)
         comm.load(hdr + " chunkbytes=65536 instances=2 fifodepth=2 direct=1\n" + rest)
-        x = to_torch(inp.rank_input("int32", 9, rank, count), "int32")
-        win = torch.zeros(2 * count + 64, dtype=torch.int32, device="cuda:0")
+        x = to_torch(inp.rank_input("int32", 9, rank, count), "int32", f"cuda:{dev}")
+        win = torch.zeros(2 * count + 64, dtype=torch.int32, device=f"cuda:{dev}")
         comm.register(win)
         s_reg, r_reg = win[:count], win[count + 64:2 * count + 64]
         s_reg.copy_(x)
-        r_un = torch.zeros(count, dtype=torch.int32, device="cuda:0")
+        r_un = torch.zeros(count, dtype=torch.int32, device=f"cuda:{dev}")
         comm.allreduce(s_reg, r_reg)  # eager warm-up: both plans compiled outside the capture
         comm.allreduce(x, r_un)
         torch.cuda.synchronize()

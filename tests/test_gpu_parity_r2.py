@@ -1,0 +1,101 @@
+"""GPU parity of the SURVEY §8(f) rows f1 and f2 on the device.
+
+* f2: plans scheduled by the round-robin baseline (``sched=rr``)
+  give different sub-pipelines, lane lists and orders than HPDS.  A wrong order could
+  deadlock or race on the device, so they run here -- staged and direct transports,
+  register and TMA paths -- against the oracle's replay of the oracle's own RR plan.
+* f1: the paper's Fig. 16 program text (``tests/golden``) is loaded
+  verbatim (only nNodes / nGpusperNode / nRanks / GPUPerNode instantiated for 8 ranks)
+  through ``rescclLoadAlgorithm``: the C++ ResCCLang front end, planner and generated
+  kernel run it, and the result must equal the oracle's replay of its own transcription
+  of the listing (``oracle.ir.hm_allreduce``) byte for byte.
+"""
+import os
+
+import numpy as np
+import pytest
+
+import resccl_inputs as inp
+from gpu_helpers import run_virtual
+from oracle import dag, definition, hpds, ir as oir, lower, replay
+
+pytestmark = pytest.mark.gpu
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+RR_CASES = [
+    ("dbt", "allreduce", 8, {}), ("hm", "allreduce", 8, {"g": 4}), ("hm", "allgather", 8, {"g": 4}),
+    ("synth", "allgather", 8, {"seed": 0, "fanout": 2}), ("synth", "reducescatter", 8, {"seed": 1, "fanout": 3}),
+    ("ring", "allreduce", 8, {}),
+]
+
+
+def _rr_expect(g, xs, dtype, count, cb, inst, K, direct):
+    edges, _ = dag.build_dag(g)
+    pl = lower.lower(g, "pair", Pr=hpds.round_robin(g, edges, "pair"), direct=direct)
+    return replay.replay(pl, xs, dtype, count, chunk_bytes=cb, instances=inst, K=K)
+
+
+def _check(outs, exp):
+    for r in range(len(outs)):
+        assert np.array_equal(outs[r].view(np.uint8), exp[r].view(np.uint8)), f"rank {r}"
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("name,coll,n,kw", RR_CASES)
+@pytest.mark.parametrize("direct", [0, 1])
+def test_round_robin_plans_bit_exact(name, coll, n, kw, direct):
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    g = oir.generate(name, coll, n, **kw)
+    count = 3 * 4096 + 77
+    for k, v in dict(sched="rr", chunkbytes=4096, instances=2, fifodepth=2, direct=direct).items():
+        g.extra[k] = str(v)
+    m = count * n if coll == "reducescatter" else count
+    xs = inp.all_inputs("bfloat16", 21, n, m)
+    outs, info, err = run_virtual(R, g.to_text(), coll, xs, "bfloat16", count)
+    assert err == 0 and info["sched"] == "rr"
+    _check(outs, _rr_expect(g, xs, "bfloat16", count, 4096, 2, 2, bool(direct)))
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("name,coll,kw", [("dbt", "allreduce", {}), ("hm", "allreduce", {"g": 4}),
+                                          ("synth", "reducescatter", {"seed": 0, "fanout": 2})])
+def test_round_robin_plans_tma_path(name, coll, kw):
+    """Instance slices above tmamin: the TMA lane engine runs the RR lane lists."""
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    n = 8
+    g = oir.generate(name, coll, n, **kw)
+    count = (2 << 20) + 4099
+    for k, v in dict(sched="rr", chunkbytes=1 << 20, instances=2, fifodepth=2, direct=1).items():
+        g.extra[k] = str(v)
+    m = count * n if coll == "reducescatter" else count
+    xs = inp.all_inputs("float32", 22, n, m)
+    outs, info, err = run_virtual(R, g.to_text(), coll, xs, "float32", count)
+    assert err == 0
+    _check(outs, _rr_expect(g, xs, "float32", count, 1 << 20, 2, 2, True))
+
+
+def _fig16_text(n_nodes, gpn):
+    src = open(os.path.join(GOLD, "fig16_hm_allreduce.py.txt")).read()
+    src = src.replace("nRanks =32", f"nRanks ={n_nodes * gpn}").replace("GPUPerNode =8", f"GPUPerNode ={gpn}")
+    src = src.replace("    nNodes = 4\n", f"    nNodes = {n_nodes}\n")
+    return src.replace("    nGpusperNode = 8\n", f"    nGpusperNode = {gpn}\n")
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("dtype", ["bfloat16", "int32"])
+def test_fig16_program_text_on_gpu(dtype):
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    text = _fig16_text(2, 4)
+    assert text.lstrip("#").find("def ResCCLAlgo") >= 0
+    n, count = 8, (3 << 20) + 1001
+    xs = inp.all_inputs(dtype, 23, n, count)
+    outs, info, err = run_virtual(R, text, "allreduce", xs, dtype, count)
+    assert err == 0
+    assert info["instances"] == 4 and info["nwarps"] == 16   # nChannels=4, nWarps=16 (Fig. 16 header)
+    assert info["ctas"] == [4] * n                            # Table 3 Topo1: 8 lanes = 4 duplex CTAs
+    g = oir.hm_allreduce(2, 4)
+    exp = replay.replay(lower.lower(g), xs, dtype, count, chunk_bytes=1 << 20, instances=4, K=4)
+    _check(outs, exp)
+    if dtype == "int32":
+        _check(outs, definition.allreduce(xs, "int32"))
