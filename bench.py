@@ -146,9 +146,17 @@ class ClockSampler:
 
 # ---------------------------------------------------------------------------- CPU oracle leg
 
+def host_cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:  # noqa: BLE001
+        return os.cpu_count() or 1
+
+
 def cpu_oracle_sample(algo: str, n: int, dtype: str, budget_s: float = 12.0):
-    """Time the oracle (schedule replay, as it stands) on a bounded sample of the same
-    workload; returns (busBW-equivalent GB/s, seconds per call, sample description)."""
+    """Time the oracle's Python schedule replay (the blocking FIFO simulator, as it
+    stands) on a bounded sample of the same workload; returns (busBW-equivalent GB/s,
+    seconds per call, sample description)."""
     import resccl_inputs as inp
     from oracle import ir as oir, lower, replay
     g = oir.generate(algo, "allreduce", n, **({"g": 4} if algo == "hm" else {}))
@@ -165,51 +173,89 @@ def cpu_oracle_sample(algo: str, n: int, dtype: str, budget_s: float = 12.0):
     dt = (time.perf_counter() - t0) / reps
     S = count * ELT[dtype]
     bus = S / dt * 2 * (n - 1) / n / 1e9
-    return bus, dt, f"{algo} allreduce, {n} ranks x {S >> 20} MiB {dtype}, {reps} replay(s), 1 thread"
+    return bus, dt, f"{algo} allreduce, {n} ranks x {S >> 20} MiB {dtype}, {reps} replay(s), 1 thread (Python)"
 
 
-def _oracle_worker(a):
-    algo, n, dtype, budget = a
-    return cpu_oracle_sample(algo, n, dtype, budget_s=budget)
+def c1_replay_seconds(reps: int = 3) -> float:
+    """BASELINE configs[0] -- ring AllReduce of 4096 fp32, 2 ranks, 1 TB, 4 chunks -- as
+    the oracle's Python schedule replay: seconds per replay."""
+    import resccl_inputs as inp
+    from oracle import ir as oir, lower, replay
+    g = oir.ring_allreduce(2)
+    pl = lower.lower(g)
+    xs = inp.all_inputs("float32", 0, 2, 4096)
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        replay.replay(pl, xs, "float32", 4096, chunk_bytes=4096, instances=1, K=4)
+    return (time.perf_counter() - t0) / reps
 
 
-def cpu_oracle_all_cores(algo: str, n: int, dtype: str, budget_s: float = 8.0):
-    """The same oracle sample run concurrently in one process per host core (SURVEY d6:
-    1 thread and all cores); returns (aggregate GB/s, cores, mean s per call).  A broken
-    or slow worker raises (bounded wait) instead of hanging the bench."""
-    import concurrent.futures as cf
-    import multiprocessing as mp
-    procs = max(1, min(os.cpu_count() or 1, 32))
-    with cf.ProcessPoolExecutor(procs, mp_context=mp.get_context("spawn")) as ex:
-        futs = [ex.submit(_oracle_worker, (algo, n, dtype, budget_s)) for _ in range(procs)]
-        res = [f.result(timeout=budget_s * 4 + 120) for f in futs]
-    return sum(r[0] for r in res), procs, statistics.mean(r[1] for r in res)
+def host_workload(n: int, count: int, dtype: str, seed: int = 0):
+    """Synthetic host buffers with the bench workload's shape (uniform [-1, 1), the d2
+    value distribution) for the CPU legs."""
+    import numpy as np
+    rng = np.random.default_rng(seed)
+    out = []
+    for _ in range(n):
+        f = (rng.random(count, dtype=np.float32) * 2 - 1)
+        if dtype == "bfloat16":
+            out.append((f.view(np.uint32) >> 16).astype(np.uint16))
+        elif dtype == "float16":
+            out.append(f.astype(np.float16))
+        elif dtype == "float32":
+            out.append(f)
+        else:
+            out.append((f * (1 << 20)).astype(np.int32))
+    return out
+
+
+def cpu_fast_replay(algo: str, n: int, dtype: str, xs, count: int, threads: int, reps: int = 1):
+    """The oracle's C++ fast replay (oracle/fastreplay.cc) of the WHOLE bench workload;
+    returns (busBW-equivalent GB/s, seconds per call)."""
+    import numpy as np
+    from oracle import fastreplay, ir as oir
+    g = oir.generate(algo, "allreduce", n, **({"g": 4} if algo == "hm" else {}))
+    outs = [np.empty_like(x) for x in xs]
+    fastreplay.replay_full(g, xs, dtype, count, threads=threads, outputs=outs)  # warm (pages, lib load)
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        fastreplay.replay_full(g, xs, dtype, count, threads=threads, outputs=outs)
+    dt = (time.perf_counter() - t0) / reps
+    S = count * ELT[dtype]
+    return S / dt * 2 * (n - 1) / n / 1e9, dt
 
 
 def reference_impl(args):
-    """--impl reference: the oracle timed on the host cores (tier framing)."""
+    """--impl reference: the oracle timed on the host cores (tier framing).  A step = the
+    C++ fast replay of the same workload as the ResCCL arm (same algorithm, ranks, bytes
+    per rank, dtype) on every host core."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     n = args.vranks if args.gpus == 1 else args.gpus
-    vals = []
+    count = int(args.size_mb * (1 << 20)) // ELT[args.dtype]
+    S = count * ELT[args.dtype]
+    cores = host_cores()
+    xs = host_workload(n, count, args.dtype)
     for _ in range(args.warmup):
-        cpu_oracle_sample(args.algo, n, args.dtype, budget_s=0.0)
-    t_all = []
+        cpu_fast_replay(args.algo, n, args.dtype, xs, count, cores, reps=1)
+    vals, t_all = [], []
     for _ in range(args.steps):
-        bus, dt, desc = cpu_oracle_sample(args.algo, n, args.dtype, budget_s=0.0)
+        bus, dt = cpu_fast_replay(args.algo, n, args.dtype, xs, count, cores, reps=1)
         vals.append(bus)
         t_all.append(dt)
-    value = statistics.mean(vals)
+    value = S * args.steps / sum(t_all) * 2 * (n - 1) / n / 1e9
+    desc = (f"{args.algo} allreduce, {n} ranks x {S >> 20} MiB {args.dtype} (the whole workload), C++ fast "
+            f"replay (oracle/fastreplay.cc), {cores} threads")
     line = {
         "impl": "reference", "metric": "allreduce busBW", "value": round(value, 4), "unit": "GB/s",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(1e3 * statistics.mean(t_all), 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": {"bfloat16": "bf16"}.get(args.dtype, args.dtype),
         "data": "synthetic",
-        "config": {"workload": f"{args.algo} allreduce, {n} ranks, CPU oracle schedule replay "
-                               f"(bounded sample: 4 MiB per rank)", "nranks": n},
-        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+        "config": {"workload": f"{args.algo} allreduce, {n} ranks, {S >> 20} MiB per rank, CPU oracle schedule "
+                               f"replay on the host cores", "nranks": n, "bytes_per_rank": S},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": cores, "kind": "oracle",
                          "sample": desc},
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -478,16 +524,26 @@ def main():
 
     cpu = None
     if not args.no_cpu_baseline and not multi:
-        bus_cpu, dt_cpu, desc = cpu_oracle_sample(args.algo, n, args.dtype)
-        cpu = {"value": round(bus_cpu, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc,
-               "s_per_call": round(dt_cpu, 3)}
-        try:
-            agg, procs, dt_all = cpu_oracle_all_cores(args.algo, n, args.dtype)
-            cpu["all_cores"] = {"value": round(agg, 4), "unit": "GB/s", "cores": procs,
-                                "s_per_call": round(dt_all, 3),
-                                "sample": "the same sample, one oracle process per host core"}
-        except Exception as e:  # noqa: BLE001 -- the single-thread figure stands
-            cpu["all_cores"] = {"error": str(e)[:200]}
+        # the oracle as it stands, on the host cores: the C++ fast replay
+        # of the whole workload (these very inputs, copied to the host) at all cores and at
+        # 1 thread, the Python blocking replay on a bounded sample, and C1 in seconds
+        import numpy as np
+        xs_host = [(sends[r].cpu().view(torch.int16).numpy().view(np.uint16) if args.dtype == "bfloat16"
+                    else sends[r].cpu().numpy()) for r in my_ranks]
+        cores = host_cores()
+        bus_all, dt_all = cpu_fast_replay(args.algo, n, args.dtype, xs_host, count, cores, reps=2)
+        bus_1, dt_1 = cpu_fast_replay(args.algo, n, args.dtype, xs_host, count, 1, reps=1)
+        del xs_host
+        bus_py, dt_py, desc_py = cpu_oracle_sample(args.algo, n, args.dtype, budget_s=6.0)
+        cpu = {"value": round(bus_all, 4), "unit": "GB/s", "cores": cores, "kind": "oracle",
+               "sample": (f"the whole workload ({n} ranks x {S >> 20} MiB {args.dtype}, this run's inputs): "
+                          f"C++ fast replay (oracle/fastreplay.cc), {cores} threads, 2 calls"),
+               "s_per_call": round(dt_all, 3),
+               "one_thread": {"value": round(bus_1, 4), "unit": "GB/s", "cores": 1, "s_per_call": round(dt_1, 3)},
+               "python_replay": {"value": round(bus_py, 4), "unit": "GB/s", "cores": 1,
+                                 "s_per_call": round(dt_py, 3), "sample": desc_py},
+               "c1_replay_s": round(c1_replay_seconds(), 4),
+               "c1": "BASELINE configs[0]: ring AllReduce 4096 fp32, 2 ranks, 1 TB, 4 chunks (Python replay)"}
 
     # SMs the kernel occupies: its CTAs (one or two per SM, by block size) spread over the SMs
     n_sm = torch.cuda.get_device_properties(dev).multi_processor_count

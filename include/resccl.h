@@ -173,6 +173,22 @@ rescclResult_t rescclGetPlanInfo(rescclAlgo_t algo, char* json, size_t* len);
  * RESCCL_TRACE=1) and the launch finished (synchronise the stream first). */
 rescclResult_t rescclGetTbUtilization(rescclAlgo_t algo, char* json, size_t* len);
 
+/* Phase records of the last launch of `algo` (where a hop's time
+ * goes).  Requires the algorithm loaded with phase=1.  Every lane leader writes one
+ * record per (primitive, micro-batch) into device memory with %globaltimer stamps;
+ * this call synchronises the device and copies them out as u64 words:
+ *   [0] blocks, [1] first global block, [2] records per (block, lane) P, [3] instances,
+ *   then for block b (launch-relative) and lane l (0 send, 1 recv) P records of 8 words
+ *   at 4 + (2b + l)·8P.  Record 0 = lane header {entry ns, exit ns, records, rank, cta,
+ *   instance}; record k >= 1 = {prim << 32 | mb << 8 | kind, t0, t1, t2, t3, t4},
+ *   kind 0 register path (t0 start, t1 dependencies met, t2 flag / credit met, t3 data
+ *   moved, t4 posted), 1 flag-only primitive (t0 start of wait, t1 dependencies met /
+ *   readable or writable posted, t2 peer's payload seen, t4 posted), 2 TMA engine
+ *   (t0 previous post, t1 ready, t3 stores complete, t4 posted); 0 = not recorded.
+ * buf NULL: *len = bytes needed.  Ownership: the caller owns buf.  InvalidUsage when the
+ * algorithm was not loaded with phase=1 or has not run; CudaError on copy failure. */
+rescclResult_t rescclGetPhaseTrace(rescclAlgo_t algo, void* buf, size_t* len);
+
 /* ------------------------------------------------------------------ collectives */
 
 /* out_r[i] = sum_k in_k[i].  sendbuf/recvbuf: count elements each. */

@@ -43,6 +43,7 @@ EXPORTS = [
     "rescclCommGetHandle", "rescclCommConnect", "rescclCommInit", "rescclCommInitAll",
     "rescclCommDestroy", "rescclCommRank", "rescclCommCount", "rescclCommGetAsyncError",
     "rescclLoadAlgorithm", "rescclSetActiveAlgorithm", "rescclGetPlanInfo", "rescclGetTbUtilization",
+    "rescclGetPhaseTrace",
     "rescclAllReduce",
     "rescclAllGather", "rescclReduceScatter", "rescclGenerateIr", "rescclPlanIr",
     "rescclCodegenIr", "rescclCompileIr", "rescclCheckDeadlock", "rescclParseResCCLang", "rescclProfilePlanner",
@@ -68,6 +69,7 @@ _SIGS = {
     "rescclSetActiveAlgorithm": (_i, [_vp, _vp]),
     "rescclGetPlanInfo": (_i, [_vp, _c.c_char_p, _c.POINTER(_sz)]),
     "rescclGetTbUtilization": (_i, [_vp, _c.c_char_p, _c.POINTER(_sz)]),
+    "rescclGetPhaseTrace": (_i, [_vp, _vp, _c.POINTER(_sz)]),
     "rescclAllReduce": (_i, [_vp, _vp, _sz, _i, _i, _vp, _vp]),
     "rescclAllGather": (_i, [_vp, _vp, _sz, _i, _vp, _vp]),
     "rescclReduceScatter": (_i, [_vp, _vp, _sz, _i, _i, _vp, _vp]),
@@ -275,6 +277,15 @@ def rescclGetTbUtilization(algo: int) -> dict:
     buf = _c.create_string_buffer(n.value)
     _check(_lib.rescclGetTbUtilization(algo, buf, _c.byref(n)), "rescclGetTbUtilization")
     return json.loads(buf.value.decode())
+
+
+def rescclGetPhaseTrace(algo: int) -> List[int]:
+    """Raw u64 words of the last launch's phase records (layout: include/resccl.h)."""
+    n = _sz(0)
+    _check(_lib.rescclGetPhaseTrace(algo, None, _c.byref(n)), "rescclGetPhaseTrace")
+    buf = (_c.c_ulonglong * (n.value // 8))()
+    _check(_lib.rescclGetPhaseTrace(algo, buf, _c.byref(n)), "rescclGetPhaseTrace")
+    return list(buf)
 
 
 def rescclAllReduce(sendbuf: int, recvbuf: int, count: int, dtype: int, op: int, comm: int,

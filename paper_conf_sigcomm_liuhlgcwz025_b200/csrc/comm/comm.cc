@@ -38,6 +38,7 @@ namespace {
 
 using namespace resccl;
 constexpr int kMaxR = 32;
+#define RESCCL_PH_MAX_HOST 96  // = RESCCL_PH_MAX (resccl_device.cuh): phase records per (block, lane)
 
 // host mirror of rdev::KArgs (resccl_device.cuh)
 struct KArgs {
@@ -54,6 +55,7 @@ struct KArgs {
   unsigned long long* trace;
   unsigned long long epoch;
   unsigned long long* epochs;  // device-side epochs {mb_base, epoch, CTAs done}, or null
+  unsigned long long* phase;   // phase=1: per-(block, lane) phase records (device memory), or null
 };
 
 thread_local std::string g_last_error;
@@ -137,6 +139,7 @@ struct Options {
                           // (192 KiB smem per CTA, one CTA per SM) moves 1.4x the bytes per SM of 12 KiB x 4
   int tma_stages = 2;
   int trace = 0;
+  int phase = 0;     // %globaltimer phase records per (primitive, micro-batch) (rescclGetPhaseTrace)
   int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
   int direct = 0;    // direct transport (R23): virtual ranks / single-process only
   int l2hint = 1;
@@ -192,6 +195,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "tmatile") o.tma_tile = (int)to_long(v, k);
   else if (k == "tmastages") o.tma_stages = (int)to_long(v, k);
   else if (k == "trace") o.trace = (int)to_long(v, k);
+  else if (k == "phase") o.phase = (int)to_long(v, k);
   else if (k == "l2hint") o.l2hint = (int)to_long(v, k);
   else if (k == "prefetch") o.prefetch = (int)to_long(v, k);
   else if (k == "tmamin") o.tma_min = (int)to_long(v, k);
@@ -355,6 +359,8 @@ struct AlgoShared {
   unsigned long long* trace_dev = nullptr;
   int trace_blocks = 0;                // blocks covered by the last traced launch
   int trace_block_base = 0;
+  unsigned long long* phase_dev = nullptr;  // phase=1: records of the last launch (device memory)
+  int phase_blocks = 0, phase_block_base = 0, phase_dev_id = 0;
   std::shared_ptr<AlgoShared> twin;    // multi-process direct plan: staged plan for unregistered buffers
   char* region_alloc = nullptr;
   int64_t region_off = 0;              // multi-process: offset inside the arena
@@ -523,6 +529,7 @@ CodegenOpts codegen_opts(const Options& o) {
   co.tma_tile = o.tma_tile;
   co.tma_stages = o.tma_stages;
   co.trace = o.trace;
+  co.phase = o.phase;
   co.l2hint = o.l2hint;
   co.prefetch = o.prefetch;
   co.tma_min = o.tma_min;
@@ -665,6 +672,19 @@ unsigned long long* trace_buffer(AlgoShared& a, int blocks, int block_base) {
   return a.trace_dev;
 }
 
+// phase=1: the record area of this launch, cleared on the launch stream
+unsigned long long* phase_buffer(AlgoShared& a, int blocks, int block_base, int dev, cudaStream_t s) {
+  if (!a.opt.phase) return nullptr;
+  const size_t per = (size_t)RESCCL_PH_MAX_HOST * 8 * sizeof(unsigned long long);
+  const size_t bytes = (size_t)a.lay.total_pairs * a.opt.instances * 2 * per;
+  if (!a.phase_dev) cuda_check(cudaMalloc((void**)&a.phase_dev, bytes), "cudaMalloc(phase)");
+  cuda_check(cudaMemsetAsync(a.phase_dev, 0, bytes, s), "cudaMemsetAsync(phase)");
+  a.phase_blocks = blocks;
+  a.phase_block_base = block_base;
+  a.phase_dev_id = dev;
+  return a.phase_dev;
+}
+
 // connected window containing [p, p + bytes), or -1
 int find_window(const rescclComm* comm, const void* p, size_t bytes) {
   for (size_t w = 0; w < comm->windows.size(); ++w) {
@@ -726,6 +746,7 @@ void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const vo
   ka.err = comm->err_dev;
   ka.timeout_ns = timeout_ns();
   ka.trace = trace_buffer(a, a.lay.ctas[comm->rank] * a.opt.instances, ka.block_base);
+  ka.phase = phase_buffer(a, a.lay.ctas[comm->rank] * a.opt.instances, ka.block_base, comm->dev, s);
   if (a.opt.devepoch) ka.epochs = algo->dev_epochs[ap == algo->s.get() ? 0 : 1];
   const bool use_tma = a.opt.tma && g.Mi * elt_size(c.dt) >= a.opt.tma_min;
   Kern& k = get_kernel(a, c.dt, c.op, comm->rank, comm->rank + 1, false, use_tma);
@@ -757,6 +778,7 @@ void group_launch(Group* G, Pending& p) {
   ka.err = G->err_dev;
   ka.timeout_ns = timeout_ns();
   ka.trace = trace_buffer(a, a.lay.total_pairs * a.opt.instances, 0);
+  ka.phase = phase_buffer(a, a.lay.total_pairs * a.opt.instances, 0, G->dev, p.streams.back());
   if (a.opt.devepoch) ka.epochs = a.dev_epochs;
   const bool use_tma = a.opt.tma && g.Mi * elt_size(c.dt) >= a.opt.tma_min;
   Kern& k = get_kernel(a, c.dt, c.op, 0, G->nranks, true, use_tma);
@@ -1726,6 +1748,8 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
         kv.second->kernels.clear();
         if (kv.second->region_alloc) cudaFree(kv.second->region_alloc);
         if (kv.second->dev_epochs) cudaFree(kv.second->dev_epochs);
+        if (kv.second->phase_dev) cudaFree(kv.second->phase_dev);
+        if (kv.second->trace_host) cudaFreeHost(kv.second->trace_host);
       }
       for (auto e : G->events) cudaEventDestroy(e);
       G->hcopy.release();
@@ -1741,9 +1765,12 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
         if (e) cudaFree(e);
       if (a->s.use_count() == 1)
         for (AlgoShared* x : {a->s.get(), a->s->twin.get()})
-          if (x)
+          if (x) {
             for (auto& k : x->kernels)
               if (k.second.mod) driver().ModuleUnload(k.second.mod);
+            if (x->phase_dev) cudaFree(x->phase_dev);
+            if (x->trace_host) cudaFreeHost(x->trace_host);
+          }
     }
     for (int q = 0; q < (int)comm->peer_opened.size(); ++q)
       if (comm->peer_opened[q]) cudaIpcCloseMemHandle(comm->peer_arena[q]);
@@ -1801,6 +1828,35 @@ rescclResult_t rescclGetPlanInfo(rescclAlgo_t algo, char* json, size_t* len) {
   if (!algo) fail(rescclInvalidArgument, "algo is NULL");
   if (algo->s->json.empty()) algo->s->json = info_json(*algo->s);
   write_out(algo->s->json, json, len);
+  API_END
+}
+
+rescclResult_t rescclGetPhaseTrace(rescclAlgo_t algo, void* buf, size_t* len) {
+  API_BEGIN
+  if (!algo) fail(rescclInvalidArgument, "algo is NULL");
+  if (!len) fail(rescclInvalidArgument, "len is NULL");
+  AlgoShared& a = *algo->s;
+  if (!a.opt.phase || !a.phase_dev) fail(rescclInvalidUsage, "no phase trace: load with phase=1 and run");
+  const size_t per = (size_t)RESCCL_PH_MAX_HOST * 8;
+  const size_t words = 4 + (size_t)a.phase_blocks * 2 * per;
+  if (!buf) {
+    *len = words * sizeof(unsigned long long);
+    return rescclSuccess;
+  }
+  if (*len < words * sizeof(unsigned long long)) {
+    *len = words * sizeof(unsigned long long);
+    fail(rescclInvalidArgument, "buffer too small");
+  }
+  auto* out = (unsigned long long*)buf;
+  out[0] = (unsigned long long)a.phase_blocks;
+  out[1] = (unsigned long long)a.phase_block_base;
+  out[2] = (unsigned long long)RESCCL_PH_MAX_HOST;
+  out[3] = (unsigned long long)a.opt.instances;
+  cuda_check(cudaSetDevice(a.phase_dev_id), "cudaSetDevice");
+  cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
+  cuda_check(cudaMemcpy(out + 4, a.phase_dev, (words - 4) * sizeof(unsigned long long), cudaMemcpyDeviceToHost),
+             "cudaMemcpy(phase)");
+  *len = words * sizeof(unsigned long long);
   API_END
 }
 

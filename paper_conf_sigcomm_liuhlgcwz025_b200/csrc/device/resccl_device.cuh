@@ -33,6 +33,13 @@
 #ifndef RESCCL_TRACE
 #define RESCCL_TRACE 0
 #endif
+// RESCCL_PHASE: per-(primitive, micro-batch) %globaltimer phase records of every lane
+// leader (device memory, read back by rescclGetPhaseTrace): where a hop's time goes
+// (dependency wait, flag / credit wait, data movement, fence + post).
+#ifndef RESCCL_PHASE
+#define RESCCL_PHASE 0
+#endif
+#define RESCCL_PH_MAX 96   // records per (block, lane); record 0 = lane header
 
 namespace rdev {
 
@@ -60,6 +67,7 @@ struct KArgs {
   u64* epochs;                        // device-side epochs (graph-capturable launches), or null:
                                       // {mb_base, epoch, CTAs done}; the kernel reads the first two
                                       // instead of the fields above, the last CTA advances them
+  u64* phase;                         // RESCCL_PHASE: RESCCL_PH_MAX x 8 u64 per (block, lane), or null
 };
 
 // Device-side epochs: every CTA takes this launch's micro-batch base and call epoch from
@@ -566,6 +574,9 @@ struct Lane {
   u32 ring0;                 // RESCCL_RING: first stage of this lane's private ring
   u32 cpar;                  // RESCCL_RING (leader): comp-barrier phase parity per ring slot
   u64 wait_ns;               // RESCCL_TRACE: leader time spent waiting (idle ratio, Table 3)
+  int pidx;                  // index of the running primitive in the rank's descriptor table
+  u64* ph;                   // RESCCL_PHASE: this lane's record area (null: off)
+  u32 nph;                   // RESCCL_PHASE: records written
 
   __device__ __forceinline__ void sync() const {
     asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(nthreads) : "memory");
@@ -590,6 +601,31 @@ struct Lane {
 };
 
 __device__ __forceinline__ u64* at(char* base, i64 off) { return (u64*)(base + off); }
+
+// RESCCL_PHASE record (leader only): kind 0 = blocking register path, 1 = flag-only
+// primitive, 2 = TMA lane engine; t[0..4] as documented at each call site.
+enum : int { PhSync = 0, PhFlags = 1, PhPipe = 2 };
+__device__ __forceinline__ void ph_rec(Lane& L, int kind, int j, u64 t0, u64 t1, u64 t2, u64 t3, u64 t4) {
+#if RESCCL_PHASE
+  if (!L.ph || L.nph + 1 >= RESCCL_PH_MAX) return;
+  u64* r = L.ph + 8 * (size_t)(++L.nph);
+  r[0] = ((u64)(u32)L.pidx << 32) | ((u64)(u32)j << 8) | (u64)kind;
+  r[1] = t0;
+  r[2] = t1;
+  r[3] = t2;
+  r[4] = t3;
+  r[5] = t4;
+#else
+  (void)L; (void)kind; (void)j; (void)t0; (void)t1; (void)t2; (void)t3; (void)t4;
+#endif
+}
+__device__ __forceinline__ u64 ph_now() {
+#if RESCCL_PHASE
+  return globaltimer();
+#else
+  return 0;
+#endif
+}
 
 template <int COLL>
 __device__ __forceinline__ i64 chunk_len(const KArgs& a, int c) {
@@ -756,10 +792,15 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
   for (int j = 0; j < a.n_mb; ++j) {
     const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
     const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
+    // phase record: t0 start, t1 local dependencies met, t2 flag / credit met, t3 data
+    // moved (lane barrier passed), t4 posted (fence + flag stores issued)
+    u64 ph0 = 0, ph1 = 0, ph2 = 0;
     if (L.tid == 0) {
+      ph0 = ph_now();
       bool ok = true;
       for (int k = 0; k < d.ndeps && ok; ++k)
         ok = L.wait_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, j));
+      ph1 = ph_now();
       if (ok && Kind<F>::push_recv) post_writable<F>(a, d, p, j);
       if (ok && (F & kRecv)) ok = L.wait_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1);
       if (ok && (F & kSend)) {
@@ -770,6 +811,7 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
         }
       }
       if (!ok) *L.abort_flag = 1;
+      ph2 = ph_now();
     }
     L.sync();
     if (*L.abort_flag) return false;
@@ -784,7 +826,11 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
                                    : nullptr;
     move<T, OP, Kind<F>::mf, 4>(hi - lo, Aj, Bj, D1j, D2j, L.tid, L.nthreads);
     L.sync();
-    if (L.tid == 0) post_mb<F>(a, d, p, j);
+    if (L.tid == 0) {
+      const u64 ph3 = ph_now();
+      post_mb<F>(a, d, p, j);
+      ph_rec(L, PhSync, j, ph0, ph1, ph2, ph3, ph_now());
+    }
   }
   return true;
 }
@@ -939,6 +985,11 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   const u64 pol_last = policy_evict_last();
   int pf = 0;                 // next micro-batch whose local slice gets an L2 prefetch
   int wp = 0;                 // push receiver (drecv_d): micro-batches posted "writable"
+#if RESCCL_PHASE
+  // phase records: t0 previous post (or entry), t1 micro-batch ready (dependencies, flag,
+  // credit), t3 every store of it complete, t4 posted
+  u64 ph_rdy[8], ph_w = ph_now();
+#endif
   while (pj < nmb) {
     bool prog = false;
     if (Kind<F>::push_recv) {  // post "writable" as far ahead as the dependencies allow
@@ -966,6 +1017,9 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
     // (1) readiness of the micro-batch the load cursor needs
     if (rj < nmb && rj == lj && (!Kind<F>::push_recv || rj < wp) && mb_ready<F>(L, d, p, rj)) {
       fence_proxy_async();  // generic-proxy data (acquired) -> async-proxy reads
+#if RESCCL_PHASE
+      ph_rdy[rj & 7] = ph_now();
+#endif
       ++rj;
       prog = true;
     }
@@ -1140,7 +1194,14 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
                            pD1 ? pD1 + e0 * T::kSize : nullptr, D2j, e);
       }
       fence_proxy_async();
+#if RESCCL_PHASE
+      const u64 ph3 = ph_now();
+#endif
       post_mb<F>(a, d, p, pj);
+#if RESCCL_PHASE
+      ph_rec(L, PhPipe, pj, ph_w, ph_rdy[pj & 7], 0, ph3, ph_now());
+      ph_w = ph_now();
+#endif
       ++pj;
       if (pj < nmb) {
         T_p = mb_tiles_m<F>(aM, aMi, plen, pj, Linst, T::kSize, lo_p, nb_p, bred);
@@ -1316,6 +1377,9 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
   int wp = 0, dj = 0;  // posted (readable / writable) / completed micro-batches
   u64 t_idle = 0;
   u32 spins = 0;
+  // phase records: t0 start of the wait, t1 dependencies met (readable / writable
+  // posted right after), t2 the peer's "written" flag seen (push receive), t4 posted
+  u64 ph_w = ph_now(), ph_dep[4] = {0, 0, 0, 0};
   while (recv ? dj < nmb : wp < nmb) {
     bool prog = false;
     if (wp < nmb) {
@@ -1323,13 +1387,17 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
       for (int k = 0; k < d.ndeps && ok; ++k)
         ok = ready_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, wp));
       if (ok) {
+        const u64 ph1 = ph_now();
         fence_release();
         if (!recv) {
           const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + wp;
           st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);
+          ph_rec(L, PhFlags, wp, ph_w, ph1, 0, 0, ph_now());
+          ph_w = ph_now();
         } else {
           const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + wp;
           st_relaxed(p.in_cred, in_seq + 1);
+          ph_dep[wp & 3] = ph1;
         }
         ++wp;
         prog = true;
@@ -1338,12 +1406,15 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
     if (recv && dj < wp) {
       const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + dj;
       if (ready_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1)) {
+        const u64 ph2 = ph_now();
         fence_release();
         if (F & kSend) {  // drecv_p: the payload is in our location -> readable for the next hop
           const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * nmb + dj;
           st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);
         }
         if (d.ctr >= 0) st_relaxed(p.ctr, mb_base + dj + 1);
+        ph_rec(L, PhFlags, dj, ph_w, ph_dep[dj & 3], ph2, 0, ph_now());
+        ph_w = ph_now();
         ++dj;
         prog = true;
       }

@@ -52,6 +52,7 @@ struct CodegenOpts {
   int tma_tile = 24576;          // bytes per staged tile
   int tma_stages = 2;            // stages per lane (the CTA pool holds 2x)
   int trace = 0;                 // per-lane lifetime / wait timers (TB utilisation, Table 3)
+  int phase = 0;                 // per-(primitive, micro-batch) %globaltimer phase records
   int l2hint = 1;                // L2 evict_last on FIFO writes, evict_first on streams
   int tma_min = 32768;           // slices below this many bytes use the register path
   int backoff = 1;               // nanosleep back-off while polling flags
