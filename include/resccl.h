@@ -137,6 +137,8 @@ rescclResult_t rescclCommInitAll(rescclComm_t* comms, int ndev, const int* devli
 rescclResult_t rescclCommDestroy(rescclComm_t comm);
 rescclResult_t rescclCommRank(rescclComm_t comm, int* rank);
 rescclResult_t rescclCommCount(rescclComm_t comm, int* nranks);
+/* CUDA device of this rank (virtual ranks: the shared device).  InvalidArgument on NULL. */
+rescclResult_t rescclCommCuDevice(rescclComm_t comm, int* device);
 
 /* Device-side failures (watchdog timeout) recorded since the last call: *err is
  * rescclSuccess or rescclTimeout.  Reads host-mapped memory; never blocks. */

@@ -41,7 +41,7 @@ COLLS = {"allgather": rescclCollAllGather, "reducescatter": rescclCollReduceScat
 EXPORTS = [
     "rescclGetErrorString", "rescclGetLastError", "rescclGetVersion", "rescclCommCreate",
     "rescclCommGetHandle", "rescclCommConnect", "rescclCommInit", "rescclCommInitAll",
-    "rescclCommDestroy", "rescclCommRank", "rescclCommCount", "rescclCommGetAsyncError",
+    "rescclCommDestroy", "rescclCommRank", "rescclCommCount", "rescclCommCuDevice", "rescclCommGetAsyncError",
     "rescclLoadAlgorithm", "rescclSetActiveAlgorithm", "rescclGetPlanInfo", "rescclGetTbUtilization",
     "rescclGetPhaseTrace",
     "rescclAllReduce",
@@ -64,6 +64,7 @@ _SIGS = {
     "rescclCommDestroy": (_i, [_vp]),
     "rescclCommRank": (_i, [_vp, _c.POINTER(_i)]),
     "rescclCommCount": (_i, [_vp, _c.POINTER(_i)]),
+    "rescclCommCuDevice": (_i, [_vp, _c.POINTER(_i)]),
     "rescclCommGetAsyncError": (_i, [_vp, _c.POINTER(_i)]),
     "rescclLoadAlgorithm": (_i, [_vp, _c.c_char_p, _c.POINTER(_vp)]),
     "rescclSetActiveAlgorithm": (_i, [_vp, _vp]),

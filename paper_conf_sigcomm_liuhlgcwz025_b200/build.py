@@ -22,6 +22,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 BUILD = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "libresccl.so")
+SHIM = os.path.join(HERE, "libresccl_nccl.so")   # NCCL-symbol shim (include/resccl_nccl.h)
 CUDA = os.environ.get("CUDA_HOME", "/usr/local/cuda")
 NVCC = os.path.join(CUDA, "bin", "nvcc")
 
@@ -83,6 +84,15 @@ def build(force: bool = False, verbose: bool = False) -> str:
         cmd = ["g++", "-shared", "-o", LIB] + objs + [
             "-L", os.path.join(CUDA, "lib64"), "-lcudart_static", "-lnvrtc", "-ldl", "-lrt", "-lpthread",
             "-Wl,-rpath," + os.path.join(CUDA, "lib64"), "-Wl,--no-undefined"]
+        if verbose:
+            print(" ".join(cmd))
+        _run(cmd)
+    shim_src = os.path.join(CSRC, "shim", "nccl_shim.cc")
+    shim_hdrs = [os.path.join(ROOT, "include", "resccl_nccl.h"), os.path.join(ROOT, "include", "resccl.h")]
+    if force or _newer(SHIM, [shim_src, LIB] + shim_hdrs):
+        cmd = ["g++", "-O2", "-g", "-std=c++17", "-fPIC", "-Wall", "-shared", "-I", os.path.join(ROOT, "include"),
+               shim_src, "-o", SHIM, "-L", HERE, "-lresccl", "-ldl", "-lpthread", "-Wl,-rpath,$ORIGIN",
+               "-Wl,--no-undefined"]
         if verbose:
             print(" ".join(cmd))
         _run(cmd)

@@ -1799,6 +1799,13 @@ rescclResult_t rescclCommCount(rescclComm_t comm, int* nranks) {
   API_END
 }
 
+rescclResult_t rescclCommCuDevice(rescclComm_t comm, int* device) {
+  API_BEGIN
+  if (!comm || !device) fail(rescclInvalidArgument, "null argument");
+  *device = comm->dev;
+  API_END
+}
+
 rescclResult_t rescclCommGetAsyncError(rescclComm_t comm, rescclResult_t* err) {
   API_BEGIN
   if (!comm || !err) fail(rescclInvalidArgument, "null argument");

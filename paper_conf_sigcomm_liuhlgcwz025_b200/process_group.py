@@ -45,6 +45,7 @@ _OPS = {dist.ReduceOp.SUM: "sum", dist.ReduceOp.MAX: "max", dist.ReduceOp.MIN: "
 
 
 def _op_name(op) -> str:
+    op = getattr(op, "op", op)  # options carry a ReduceOp object; its .op is the RedOpType
     if op in _OPS:
         return _OPS[op]
     if op == dist.ReduceOp.AVG:

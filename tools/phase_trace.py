@@ -83,6 +83,7 @@ def analyse(lanes, plan, inst=0):
 
     last = max(by, key=lambda x: by[x][0]["t"][4])
     t_first = min(L["entry"] for L in lanes)
+    t0_all = t_first
     t_last = max(L["exit"] for L in lanes)
     path = []
     cur = last
@@ -100,7 +101,10 @@ def analyse(lanes, plan, inst=0):
         start = rec["t"][0]
         link = {"rank": cur[0], "prim": ranks[cur[0]]["prims"][cur[1]]["kind"], "chunk": ranks[cur[0]]["prims"][cur[1]]["chunk"],
                 "mb": cur[2], "data_ns": (rec["t"][3] - rdy) if rec["t"][3] and rdy else 0,
-                "post_ns": rec["t"][4] - (rec["t"][3] or rdy or rec["t"][4])}
+                "post_ns": rec["t"][4] - (rec["t"][3] or rdy or rec["t"][4]),
+                "t_rel_ns": [(x - t0_all) if x else None for x in rec["t"]],
+                "producers": [{"rank": pk[0], "prim": ranks[pk[0]]["prims"][pk[1]]["kind"],
+                               "post_rel_ns": by[pk][0]["t"][4] - t0_all} for pk in prods]}
         if best is not None:
             ppost = by[best][0]["t"][4]
             link["handoff_ns"] = max(0, rdy - max(ppost, start)) if rdy else 0
@@ -149,6 +153,31 @@ def main():
                 grp.allreduce(s, r)
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            # (a) back-to-back eager calls: max(host submit, GPU) per call
+            import time as _t
+            h0 = _t.perf_counter()
+            e0.record()
+            for _ in range(20):
+                grp.allreduce(s, r)
+            e1.record()
+            host_us = (_t.perf_counter() - h0) / 20 * 1e6
+            torch.cuda.synchronize()
+            loop_us = e0.elapsed_time(e1) * 1e3 / 20
+            # (b) the same call captured in a CUDA graph: GPU time per call
+            st = torch.cuda.Stream()
+            gph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gph, stream=st):
+                grp.allreduce(s, r, stream=st)
+            for _ in range(3):
+                gph.replay()
+            torch.cuda.synchronize()
+            e0.record()
+            for _ in range(20):
+                gph.replay()
+            e1.record()
+            torch.cuda.synchronize()
+            graph_us = e0.elapsed_time(e1) * 1e3 / 20
+            # (c) one traced call (the analysed one)
             e0.record()
             grp.allreduce(s, r)
             e1.record()
@@ -159,6 +188,8 @@ def main():
             lanes = decode(R.rescclGetPhaseTrace(algo))
             a = analyse(lanes, plan)
             out = {"bytes": S, "opts": OPTS, "algo": ALGO, "n": N, "event_us": round(us, 2),
+                   "eager_loop_us": round(loop_us, 2), "host_submit_us": round(host_us, 2),
+                   "graph_replay_us": round(graph_us, 2),
                    "span_us": round(a["span_ns"] / 1e3, 2), "launch_overhead_us": round(us - a["span_ns"] / 1e3, 2),
                    "critical_path": {k: round(v / 1e3, 2) for k, v in a["totals"].items()},
                    "path_links": a["path_links"], "entry_skew_us": round(a["entry_skew_ns"] / 1e3, 2),
