@@ -140,6 +140,8 @@ struct Options {
   int tma_stages = 2;
   int trace = 0;
   int phase = 0;     // %globaltimer phase records per (primitive, micro-batch) (rescclGetPhaseTrace)
+  int relay_bypass = 1;  // DESIGN R29: dependents of a flags-only push receive wait on its flag
+  int lookahead = 1;     // DESIGN R30: "writable" credits posted ahead of the lane
   int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
   int direct = 0;    // direct transport (R23): virtual ranks / single-process only
   int l2hint = 1;
@@ -196,6 +198,8 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "tmastages") o.tma_stages = (int)to_long(v, k);
   else if (k == "trace") o.trace = (int)to_long(v, k);
   else if (k == "phase") o.phase = (int)to_long(v, k);
+  else if (k == "relaybypass") o.relay_bypass = (int)to_long(v, k);
+  else if (k == "lookahead") o.lookahead = (int)to_long(v, k);
   else if (k == "l2hint") o.l2hint = (int)to_long(v, k);
   else if (k == "prefetch") o.prefetch = (int)to_long(v, k);
   else if (k == "tmamin") o.tma_min = (int)to_long(v, k);
@@ -530,6 +534,8 @@ CodegenOpts codegen_opts(const Options& o) {
   co.tma_stages = o.tma_stages;
   co.trace = o.trace;
   co.phase = o.phase;
+  co.relay_bypass = o.relay_bypass;
+  co.lookahead = o.lookahead;
   co.l2hint = o.l2hint;
   co.prefetch = o.prefetch;
   co.tma_min = o.tma_min;

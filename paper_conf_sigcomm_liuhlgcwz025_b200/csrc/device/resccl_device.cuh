@@ -557,6 +557,21 @@ __device__ __forceinline__ void move(i64 n, const char* A, const char* B, char* 
 }
 
 // ----------------------------------------------------------------------------- lane
+// RESCCL_LOOKAHEAD (DESIGN R30): a lane leader posts the "writable" credits of its
+// upcoming push receives (direct transport) as soon as their dependencies hold, from any
+// idle poll, instead of when the lane reaches them.
+#if !defined(RESCCL_K)  // no plan layout (the NVLS-only self-test): no primitives either
+#undef RESCCL_LOOKAHEAD
+#define RESCCL_LOOKAHEAD 0
+#endif
+#ifndef RESCCL_LOOKAHEAD
+#define RESCCL_LOOKAHEAD 1
+#endif
+struct Lane;
+struct PrimDesc;
+template <int U = 0>
+__device__ __noinline__ void lookahead(Lane& L);
+
 struct Lane {
   const KArgs* a;
   char* self;       // this rank's plan region
@@ -577,6 +592,14 @@ struct Lane {
   int pidx;                  // index of the running primitive in the rank's descriptor table
   u64* ph;                   // RESCCL_PHASE: this lane's record area (null: off)
   u32 nph;                   // RESCCL_PHASE: records written
+  // writable lookahead (leader): the lane's push receives in lane order (descriptor index,
+  // gate = 1 + lane index of the last earlier same-lane primitive a dropped implied
+  // dependency pointed at), the cursor (push receive wa_c, micro-batch wa_m) of the next
+  // credit to post, the lane index of the running primitive and its push-receive index
+  const PrimDesc* descs;
+  const int* wa;
+  const int* wg;
+  int wa_n, wa_c, wa_m, lpos, wai;
 
   __device__ __forceinline__ void sync() const {
     asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(nthreads) : "memory");
@@ -587,6 +610,9 @@ struct Lane {
     u64 t0 = globaltimer();
     u32 spins = 0;
     while (!ready_ge(p, target)) {
+#if RESCCL_LOOKAHEAD
+      if (wa_c < wa_n) lookahead<0>(*this);
+#endif
       if (++spins > 64) nanosleep_(32);
       if ((spins & 1023) == 0 && globaltimer() - t0 > a->timeout_ns) {
         atomicCAS(a->err, 0, kErrTimeout);
@@ -664,6 +690,12 @@ struct PrimDesc {
   i64 deps[RESCCL_MAXDEPS];
   i64 dep_n[RESCCL_MAXDEPS];
   i64 dep_pos[RESCCL_MAXDEPS];
+  // bit k: dependency k is a flag ring slot instead of a counter -- the "written" flag of
+  // a flags-only push receive (drecv / drecv_p) on this rank, awaited directly instead of
+  // the counter that receive posts once it saw the flag (relay bypass, DESIGN R29): deps[k]
+  // is then the ring's offset, the slot is (target - 1) % K, the stride per instance
+  // RESCCL_FLAGSTRIDE
+  int dep_ring;
 };
 
 // Layout constants shared by every primitive of a plan (emitted by the generator):
@@ -733,6 +765,49 @@ __device__ __forceinline__ bool bulk_reduce_prim(const char* A, const char* D1) 
 __device__ __forceinline__ u64 dep_target(const KArgs& a, const PrimDesc& d, int k, int j) {
   return (u64)d.dep_n[k] * a.mb_base + (u64)d.dep_pos[k] * a.n_mb + j + 1;
 }
+// the u64 dependency k of micro-batch j waits on (see PrimDesc::dep_ring); templates so
+// that the plan's layout macros (RESCCL_K, RESCCL_FLAGSTRIDE) are needed only when used
+template <int U = 0>
+__device__ __forceinline__ const u64* dep_ptr(char* self, int inst, const PrimDesc& d, int k, u64 target) {
+  if (d.dep_ring & (1 << k))
+    return at(self, d.deps[k] + (i64)inst * RESCCL_FLAGSTRIDE + (i64)((target - 1) % RESCCL_K) * 8);
+  return at(self, d.deps[k] + (i64)inst * 128);
+}
+template <int U = 0>
+__device__ __forceinline__ bool dep_ready(const Lane& L, const PrimDesc& d, int k, int j) {
+  const u64 t = dep_target(*L.a, d, k, j);
+  return ready_ge(dep_ptr<U>(L.self, L.inst, d, k, t), t);
+}
+
+// Post at most one "writable" credit: the next one of the lane's push receives, if the
+// lane has passed every earlier same-lane primitive it depends on (gate) and its explicit
+// dependencies hold for that micro-batch -- the same conditions the primitive itself
+// checks when the lane reaches it, so the credit only comes earlier (monotone flags: no
+// new wait edge, DESIGN R30).  Leader thread only.
+template <int U>
+__device__ __noinline__ void lookahead(Lane& L) {
+  const KArgs& a = *L.a;
+  while (L.wa_c < L.wa_n) {
+    if (L.wa_m >= a.n_mb) {
+      ++L.wa_c;
+      L.wa_m = 0;
+      continue;
+    }
+    if (L.lpos < L.wg[L.wa_c]) return;
+    const PrimDesc& d = L.descs[L.wa[L.wa_c]];
+    for (int k = 0; k < d.ndeps; ++k)
+      if (!dep_ready<U>(L, d, k, L.wa_m)) return;
+    const u64 in_seq = (u64)d.in_n * a.mb_base + (u64)d.in_pos * a.n_mb + L.wa_m;
+    fence_release();
+    st_relaxed(at(a.arena[d.in_peer], d.in_cred + (i64)L.inst * 128), in_seq + 1);
+    ++L.wa_m;
+    return;
+  }
+}
+// micro-batches of the running push receive whose "writable" is posted
+__device__ __forceinline__ int writable_posted(const Lane& L, int nmb) {
+  return L.wa_c > L.wai ? nmb : (L.wa_c == L.wai ? L.wa_m : 0);
+}
 
 __device__ __forceinline__ void slice_of(const KArgs& a, i64 len, int j, int inst, i64& lo, i64& hi) {
   lo = (i64)j * a.M + (i64)inst * a.Mi;
@@ -767,7 +842,7 @@ __device__ __forceinline__ bool mb_ready(const Lane& L, const PrimDesc& d, const
   const u64 mb_base = a.mb_base;
   if (!Kind<F>::push_recv)  // (a push receiver checked its dependencies when it posted "writable")
     for (int k = 0; k < d.ndeps; ++k)
-      if (!ready_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, j))) return false;
+      if (!dep_ready(L, d, k, j)) return false;
   if (F & kRecv) {
     const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
     if (!ready_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1)) return false;
@@ -798,10 +873,28 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
     if (L.tid == 0) {
       ph0 = ph_now();
       bool ok = true;
-      for (int k = 0; k < d.ndeps && ok; ++k)
-        ok = L.wait_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, j));
+#if RESCCL_LOOKAHEAD
+      if (Kind<F>::push_recv) {  // the lane's writable cursor posts it (R30)
+        const u64 t0 = globaltimer();
+        u32 spins = 0;
+        while (writable_posted(L, a.n_mb) <= j) {
+          lookahead(L);
+          if (writable_posted(L, a.n_mb) > j) break;
+          if (++spins > 64) nanosleep_(32);
+          if ((spins & 1023) == 0 && globaltimer() - t0 > a.timeout_ns) {
+            atomicCAS(a.err, 0, kErrTimeout);
+            ok = false;
+            break;
+          }
+        }
+      } else
+#endif
+        for (int k = 0; k < d.ndeps && ok; ++k)
+          ok = L.wait_ge(dep_ptr(L.self, L.inst, d, k, dep_target(a, d, k, j)), dep_target(a, d, k, j));
       ph1 = ph_now();
+#if !RESCCL_LOOKAHEAD
       if (ok && Kind<F>::push_recv) post_writable<F>(a, d, p, j);
+#endif
       if (ok && (F & kRecv)) ok = L.wait_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1);
       if (ok && (F & kSend)) {
         if (F & kDirect) {
@@ -993,15 +1086,24 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   while (pj < nmb) {
     bool prog = false;
     if (Kind<F>::push_recv) {  // post "writable" as far ahead as the dependencies allow
+#if RESCCL_LOOKAHEAD
+      for (int n2; wp < nmb; wp = n2) {  // through the lane's writable cursor (R30)
+        lookahead(L);
+        n2 = writable_posted(L, nmb);
+        if (n2 <= wp) break;
+        prog = true;
+      }
+#else
       while (wp < nmb) {
         bool ok = true;
         for (int k = 0; k < d.ndeps && ok; ++k)
-          ok = ready_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, wp));
+          ok = dep_ready(L, d, k, wp);
         if (!ok) break;
         post_writable<F>(a, d, p, wp);
         ++wp;
         prog = true;
       }
+#endif
     }
 #if RESCCL_PREFETCH
     // (0) keep the local operand of the next RESCCL_PREFETCH micro-batches streaming into L2
@@ -1233,6 +1335,9 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
 #if RESCCL_TRACE
       if (t_idle == 0) t_idle = globaltimer();
 #endif
+#if RESCCL_LOOKAHEAD
+      if (L.wa_c < L.wa_n) lookahead(L);
+#endif
       if (stored < issued) {
         // idle with a tile outstanding: sleep on the oldest one's barrier (it is the next
         // event the store step needs) instead of polling
@@ -1382,10 +1487,20 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
   u64 ph_w = ph_now(), ph_dep[4] = {0, 0, 0, 0};
   while (recv ? dj < nmb : wp < nmb) {
     bool prog = false;
+#if RESCCL_LOOKAHEAD
+    if (recv && wp < nmb) {  // writable credits go through the lane's cursor (R30)
+      lookahead(L);
+      const int n2 = writable_posted(L, nmb);
+      if (n2 > wp) prog = true;
+      for (; wp < n2; ++wp) ph_dep[wp & 3] = ph_now();
+    }
+    if (!recv && wp < nmb) {
+#else
     if (wp < nmb) {
+#endif
       bool ok = true;
       for (int k = 0; k < d.ndeps && ok; ++k)
-        ok = ready_ge(at(L.self, d.deps[k] + (i64)L.inst * 128), dep_target(a, d, k, wp));
+        ok = dep_ready(L, d, k, wp);
       if (ok) {
         const u64 ph1 = ph_now();
         fence_release();
@@ -1428,6 +1543,9 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
     } else {
 #if RESCCL_TRACE
       if (t_idle == 0) t_idle = globaltimer();
+#endif
+#if RESCCL_LOOKAHEAD
+      if (L.wa_c < L.wa_n) lookahead(L);
 #endif
       if (++spins > 32) nanosleep_(20);
       if ((spins & 255) == 0) {

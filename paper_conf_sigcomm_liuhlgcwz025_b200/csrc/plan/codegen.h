@@ -53,6 +53,8 @@ struct CodegenOpts {
   int tma_stages = 2;            // stages per lane (the CTA pool holds 2x)
   int trace = 0;                 // per-lane lifetime / wait timers (TB utilisation, Table 3)
   int phase = 0;                 // per-(primitive, micro-batch) %globaltimer phase records
+  int relay_bypass = 1;          // wait on a flags-only push receive's flag, not its counter (R29)
+  int lookahead = 1;             // post push receives' "writable" credits ahead of the lane (R30)
   int l2hint = 1;                // L2 evict_last on FIFO writes, evict_first on streams
   int tma_min = 32768;           // slices below this many bytes use the register path
   int backoff = 1;               // nanosleep back-off while polling flags

@@ -394,6 +394,7 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
         bool implied = std::get<0>(w) == std::get<0>(me) && std::get<1>(w) == std::get<1>(me) &&
                        std::get<2>(w) < std::get<2>(me);
         if (!implied) keep.push_back(d);
+        else fin[k].implied_max = std::max(fin[k].implied_max, std::get<2>(w));
       }
       fin[k].deps = keep;
     }

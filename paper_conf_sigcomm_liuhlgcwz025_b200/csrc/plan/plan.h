@@ -68,6 +68,9 @@ struct Prim {
   int rem_buf = BufNone;  // direct mode: buffer of the peer location a pull reads
   int rem_out = BufNone;  // direct mode: buffer of the peer location a push writes
   bool has_counter = false;
+  // lane index (in its lane's list) of the last earlier same-lane primitive a dependency
+  // on which was dropped as implied by lane order, or -1 (codegen: writable lookahead, R30)
+  int implied_max = -1;
   const char* kind_name() const;
 };
 

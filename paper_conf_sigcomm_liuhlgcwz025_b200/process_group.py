@@ -53,6 +53,19 @@ def _op_name(op) -> str:
     raise ValueError(f"ResCCL backend: unsupported reduce op {op}")
 
 
+def _as_words(t: torch.Tensor) -> torch.Tensor:
+    """A dtype-agnostic view for pure data movement (AllGather, Broadcast): 32-bit words
+    when the byte count allows, else 16-bit (carried as float16 -- moved, never added)."""
+    nbytes = t.numel() * t.element_size()
+    if t.dtype in (torch.int32, torch.float32, torch.float16, torch.bfloat16) and nbytes % 4:
+        return t
+    if nbytes % 4 == 0:
+        return t.view(torch.int32) if t.dtype != torch.int32 else t
+    if nbytes % 2 == 0:
+        return t.view(torch.float16)
+    raise ValueError(f"ResCCL backend: {t.dtype} tensor of {nbytes} bytes is not a whole number of 16-bit words")
+
+
 class _Done(dist._Work):
     """A Work whose collective is already enqueued on the caller's stream."""
 
@@ -119,7 +132,7 @@ class ResCCLProcessGroup(dist.ProcessGroup):
     def _allgather_base(self, output: torch.Tensor, input: torch.Tensor, opts=None):
         self._check(output)
         self._check(input)
-        self.comm.allgather(input, output, stream=self._stream())
+        self.comm.allgather(_as_words(input), _as_words(output), stream=self._stream())
         return self._done([output])
 
     def allgather_into_tensor_coalesced(self, outputs, inputs, opts=None):
@@ -131,7 +144,7 @@ class ResCCLProcessGroup(dist.ProcessGroup):
         for outs, inp in zip(output_tensors, input_tensors):
             self._check(inp)
             flat = torch.empty(self.size() * inp.numel(), dtype=inp.dtype, device=inp.device)
-            self.comm.allgather(inp, flat, stream=self._stream())
+            self.comm.allgather(_as_words(inp), _as_words(flat), stream=self._stream())
             for q, o in enumerate(outs):
                 o.copy_(flat[q * inp.numel():(q + 1) * inp.numel()].view_as(o))
         return self._done(output_tensors)
@@ -169,11 +182,14 @@ class ResCCLProcessGroup(dist.ProcessGroup):
             if self.rank() != root:
                 t.zero_()
             nbytes = t.numel() * t.element_size()
-            v = t.view(torch.int32) if nbytes % 4 == 0 and t.dtype != torch.int32 and t.numel() > 0 else t
-            if v.dtype in (torch.int32, torch.float32, torch.float16, torch.bfloat16):
-                self.comm.allreduce(v, v, "sum", stream=self._stream())
+            if nbytes % 4 == 0:
+                v = _as_words(t)          # integer sum of the root's words and zeros: bit-exact
+            elif t.dtype in (torch.float16, torch.bfloat16):
+                v = t                     # x + 0 = x except -0.0 -> +0.0
             else:
                 raise ValueError(f"ResCCL backend: broadcast of {t.dtype} with {nbytes} bytes is unsupported")
+            if v.numel():
+                self.comm.allreduce(v, v, "sum", stream=self._stream())
         return self._done(tensors)
 
     def barrier(self, opts=None):
