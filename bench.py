@@ -59,7 +59,7 @@ def parse():
     p.add_argument("--inplace-steps", type=int, default=10,
                    help="also time in-place calls (recv = send) -> config.inplace_busbw_gbs")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--sweep", default="1,16,64",
+    p.add_argument("--sweep", default="0.0009765625,1,16,64",
                    help="comma-separated MiB-per-rank sizes for the busBW-vs-size points reported beside the "
                         "headline (slices of the bench buffers; small points are L2-resident); '' = none")
     return p.parse_args()
@@ -454,7 +454,7 @@ def main():
         inplace_bus = round(S / (ims * 1e-3) / 1e9 * 2 * (n - 1) / n, 2)
 
     # ---- extra size sweep (busBW vs size)
-    sweep = {}
+    sweep, sweep_us = {}, {}
     if args.sweep:
         for mb in [float(x) for x in args.sweep.split(",") if x]:
             cnt = int(mb * (1 << 20)) // elt
@@ -467,17 +467,35 @@ def main():
                     (comms[0] if multi else comms[r]).allreduce(s2[r], r2[r], stream=sid)
             torch.cuda.synchronize(dev)
             barrier()
+            # device clock: the calls are captured in one CUDA graph (device-side flag epochs)
+            # and replayed, so the host's per-call submission cost (8 virtual ranks x ctypes +
+            # runtime calls, ~60 us) does not hide small-message latency
+            reps = 10
+            cs = torch.cuda.Stream(dev)
+            graph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(graph, stream=cs):
+                for _ in range(reps):
+                    for r in my_ranks:
+                        (comms[0] if multi else comms[r]).allreduce(s2[r], r2[r], stream=cs.cuda_stream)
+            graph.replay()
+            torch.cuda.synchronize(dev)
+            barrier()
             a0 = torch.cuda.Event(enable_timing=True)
             a1 = torch.cuda.Event(enable_timing=True)
-            reps = 10
-            a0.record(stream)
-            for _ in range(reps):
-                for r in my_ranks:
-                    (comms[0] if multi else comms[r]).allreduce(s2[r], r2[r], stream=sid)
-            a1.record(stream)
+            a0.record(cs)
+            with torch.cuda.stream(cs):
+                graph.replay()
+            a1.record(cs)
             torch.cuda.synchronize(dev)
             t_ms = a0.elapsed_time(a1) / reps
-            sweep[f"{mb:g}MiB"] = round(cnt * elt / (t_ms * 1e-3) / 1e9 * 2 * (n - 1) / n, 2)
+            if multi:
+                t = torch.tensor([t_ms], dtype=torch.float64)
+                torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+                t_ms = float(t.item())
+            del graph
+            lab = f"{round(mb * 1024)}KiB" if mb < 1 else f"{mb:g}MiB"
+            sweep[lab] = round(cnt * elt / (t_ms * 1e-3) / 1e9 * 2 * (n - 1) / n, 2)
+            sweep_us[lab] = round(t_ms * 1e3, 2)
 
     if rank != 0:
         if multi:
@@ -578,6 +596,8 @@ def main():
     }
     if sweep:
         line["sweep_busbw_gbs"] = sweep  # busBW vs size (BASELINE metric); not the headline value
+        line["sweep_us"] = sweep_us      # device-clock time per call (CUDA-graph replay)
+        line["sweep_timing"] = "CUDA-graph replay of 10 calls (device clock; host submission excluded)"
     print(json.dumps(line), flush=True)
     if multi:
         torch.distributed.destroy_process_group()

@@ -778,6 +778,13 @@ __device__ __forceinline__ bool dep_ready(const Lane& L, const PrimDesc& d, int 
   const u64 t = dep_target(*L.a, d, k, j);
   return ready_ge(dep_ptr<U>(L.self, L.inst, d, k, t), t);
 }
+// relaxed observation only: for waits followed by fence_release() (fence.acq_rel), which
+// acquires what was observed -- no confirming acquire load (one L2 round trip less)
+template <int U = 0>
+__device__ __forceinline__ bool dep_seen(const Lane& L, const PrimDesc& d, int k, int j) {
+  const u64 t = dep_target(*L.a, d, k, j);
+  return ld_relaxed(dep_ptr<U>(L.self, L.inst, d, k, t)) >= t;
+}
 
 // Post at most one "writable" credit: the next one of the lane's push receives, if the
 // lane has passed every earlier same-lane primitive it depends on (gate) and its explicit
@@ -795,11 +802,28 @@ __device__ __noinline__ void lookahead(Lane& L) {
     }
     if (L.lpos < L.wg[L.wa_c]) return;
     const PrimDesc& d = L.descs[L.wa[L.wa_c]];
-    for (int k = 0; k < d.ndeps; ++k)
-      if (!dep_ready<U>(L, d, k, L.wa_m)) return;
     const u64 in_seq = (u64)d.in_n * a.mb_base + (u64)d.in_pos * a.n_mb + L.wa_m;
+    u64* const cred = at(a.arena[d.in_peer], d.in_cred + (i64)L.inst * 128);
+    // every probe is a relaxed load issued before any is tested (one L2 round trip in
+    // all); the fence.acq_rel before the post acquires what they observed.  The link's
+    // credit is one monotone counter for every position on the link (push "writable" and
+    // pull "read" alike): "credit >= pos + 1" must imply every earlier position was
+    // credited, so this one waits until the previous sequence was posted (by this lane or
+    // by another lane receiving on the same link)
+    u64 v[RESCCL_MAXDEPS], tg[RESCCL_MAXDEPS];
+#pragma unroll
+    for (int k = 0; k < RESCCL_MAXDEPS; ++k)
+      if (k < d.ndeps) {
+        tg[k] = dep_target(a, d, k, L.wa_m);
+        v[k] = ld_relaxed(dep_ptr<U>(L.self, L.inst, d, k, tg[k]));
+      }
+    const u64 c = ld_relaxed(cred);
+#pragma unroll
+    for (int k = 0; k < RESCCL_MAXDEPS; ++k)
+      if (k < d.ndeps && v[k] < tg[k]) return;
+    if (c < in_seq) return;
     fence_release();
-    st_relaxed(at(a.arena[d.in_peer], d.in_cred + (i64)L.inst * 128), in_seq + 1);
+    st_relaxed(cred, in_seq + 1);
     ++L.wa_m;
     return;
   }
@@ -1336,7 +1360,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       if (t_idle == 0) t_idle = globaltimer();
 #endif
 #if RESCCL_LOOKAHEAD
-      if (L.wa_c < L.wa_n) lookahead(L);
+      if (L.wa_c < L.wa_n && stored == issued && (spins & 3) == 0) lookahead(L);  // only while data-idle
 #endif
       if (stored < issued) {
         // idle with a tile outstanding: sleep on the oldest one's barrier (it is the next
@@ -1500,7 +1524,7 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
 #endif
       bool ok = true;
       for (int k = 0; k < d.ndeps && ok; ++k)
-        ok = dep_ready(L, d, k, wp);
+        ok = dep_seen(L, d, k, wp);  // (the fence.acq_rel below acquires it)
       if (ok) {
         const u64 ph1 = ph_now();
         fence_release();
@@ -1520,7 +1544,7 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
     }
     if (recv && dj < wp) {
       const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * nmb + dj;
-      if (ready_ge(p.in_flag + (in_seq % RESCCL_K), in_seq + 1)) {
+      if (ld_relaxed(p.in_flag + (in_seq % RESCCL_K)) >= in_seq + 1) {  // (acquired by the fence below)
         const u64 ph2 = ph_now();
         fence_release();
         if (F & kSend) {  // drecv_p: the payload is in our location -> readable for the next hop

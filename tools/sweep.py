@@ -5,6 +5,8 @@
   f2     HPDS vs round-robin sub-pipelines (Fig. 10b analogue)
   nr     ring allreduce bf16 at 2 / 4 / 8 virtual ranks vs size (the metric's 2/4/8 axis), the
          bench geometry with 148 // N instances per rank (every SM busy at every N)
+  geo    DBT / HM 2x4 allreduce and synthesized AG / RS at 256 MiB under transfer-chunk,
+         instance and warp-count variants (the non-ring schedules' geometry search)
 busBW follows nccl-tests: AR 2(N-1)/N, AG/RS (N-1)/N of algBW, S = per-rank buffer
 (AG: total output; RS: total input).  Usage: python tools/sweep.py c2 [c3 c4 f2]"""
 import json
@@ -114,3 +116,11 @@ if "nr" in which:
             emit(measure("ring", "allreduce", "", dict(instances=min(64, 148 // n), chunkbytes=32 << 20, fifodepth=2,
                                                        nwarps=8, direct=BASE["direct"]), S,
                          iters=20 if S < (64 << 20) else 10, n=n))
+if "geo" in which:
+    for name, coll, g in (("dbt", "allreduce", ""), ("hm", "allreduce", "g=4"), ("synth", "allgather", "seed=0 fanout=2"),
+                          ("synth", "reducescatter", "seed=0 fanout=2")):
+        for cb in (1 << 20, 4 << 20, 8 << 20, 32 << 20):
+            for inst in (4, 8):
+                for nw in (8, 16):
+                    emit(measure(name, coll, g, dict(instances=inst, chunkbytes=cb, fifodepth=2, nwarps=nw,
+                                                     direct=BASE["direct"]), 256 << 20))
