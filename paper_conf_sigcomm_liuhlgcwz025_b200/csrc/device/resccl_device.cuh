@@ -611,7 +611,7 @@ struct Lane {
     u32 spins = 0;
     while (!ready_ge(p, target)) {
 #if RESCCL_LOOKAHEAD
-      if (wa_c < wa_n) lookahead<0>(*this);
+      if (wa_c < wa_n && (spins & 7) == 7) lookahead<0>(*this);  // rate-limited: the wait's own poll first
 #endif
       if (++spins > 64) nanosleep_(32);
       if ((spins & 1023) == 0 && globaltimer() - t0 > a->timeout_ns) {
@@ -1569,7 +1569,7 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
       if (t_idle == 0) t_idle = globaltimer();
 #endif
 #if RESCCL_LOOKAHEAD
-      if (L.wa_c < L.wa_n) lookahead(L);
+      if (L.wa_c < L.wa_n && (spins & 7) == 7) lookahead(L);  // rate-limited: the flag poll first
 #endif
       if (++spins > 32) nanosleep_(20);
       if ((spins & 255) == 0) {

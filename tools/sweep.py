@@ -117,10 +117,12 @@ if "nr" in which:
                                                        nwarps=8, direct=BASE["direct"]), S,
                          iters=20 if S < (64 << 20) else 10, n=n))
 if "geo" in which:
-    for name, coll, g in (("dbt", "allreduce", ""), ("hm", "allreduce", "g=4"), ("synth", "allgather", "seed=0 fanout=2"),
-                          ("synth", "reducescatter", "seed=0 fanout=2")):
+    # instance counts keep every launch co-resident (<= 148 CTAs of one SM each)
+    for name, coll, g, insts in (("dbt", "allreduce", "", (4, 6)), ("hm", "allreduce", "g=4", (2, 4)),
+                                 ("synth", "allgather", "seed=0 fanout=2", (2, 4)),
+                                 ("synth", "reducescatter", "seed=0 fanout=2", (2, 4))):
         for cb in (1 << 20, 4 << 20, 8 << 20, 32 << 20):
-            for inst in (4, 8):
+            for inst in insts:
                 for nw in (8, 16):
                     emit(measure(name, coll, g, dict(instances=inst, chunkbytes=cb, fifodepth=2, nwarps=nw,
                                                      direct=BASE["direct"]), 256 << 20))
