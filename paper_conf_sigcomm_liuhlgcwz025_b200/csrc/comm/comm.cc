@@ -141,7 +141,7 @@ struct Options {
   int trace = 0;
   int phase = 0;     // %globaltimer phase records per (primitive, micro-batch) (rescclGetPhaseTrace)
   int relay_bypass = 1;  // DESIGN R29: dependents of a flags-only push receive wait on its flag
-  int lookahead = 1;     // DESIGN R30: "writable" credits posted ahead of the lane
+  int lookahead = 1;     // DESIGN R30: "writable" credits posted ahead of the lane (1: TMA variant, 2: both)
   int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
   int direct = 0;    // direct transport (R23): virtual ranks / single-process only
   int l2hint = 1;
@@ -561,6 +561,10 @@ Kern& get_kernel(AlgoShared& a, rescclDataType_t dt, rescclRedOp_t op, int lo, i
   co.rank_hi = hi;
   co.gpu_scope = gpu_scope;
   co.tma = use_tma ? a.opt.tma : 0;
+  // writable lookahead (R30): 1 = in the TMA-engine variant only (large slices, where it
+  // measured +2-4% at 16-64 MiB; in the latency-bound register-path variant its extra
+  // probes and fences cost more than the early credits save), 2 = in both variants
+  co.lookahead = a.opt.lookahead >= 2 || (a.opt.lookahead == 1 && use_tma) ? 1 : 0;
   co.exit_barrier = a.opt.direct && !gpu_scope;
   std::string src = codegen(a.plan, a.lay, co);
   if (const char* dump = getenv("RESCCL_DUMP_SRC")) {  // debugging aid: write the generated source
