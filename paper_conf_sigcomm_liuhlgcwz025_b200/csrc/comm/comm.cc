@@ -671,7 +671,7 @@ void fill_geometry(KArgs& ka, const Geometry& g, size_t count) {
 unsigned long long* trace_buffer(AlgoShared& a, int blocks, int block_base) {
   if (!a.opt.trace) return nullptr;
   if (!a.trace_host) {
-    size_t bytes = (size_t)a.lay.total_pairs * a.opt.instances * 2 * 4 * sizeof(unsigned long long);
+    size_t bytes = (size_t)a.lay.total_pairs * a.opt.instances * 2 * 8 * sizeof(unsigned long long);
     cuda_check(cudaHostAlloc((void**)&a.trace_host, bytes, cudaHostAllocMapped | cudaHostAllocPortable),
                "cudaHostAlloc(trace)");
     memset(a.trace_host, 0, bytes);
@@ -1884,8 +1884,8 @@ rescclResult_t rescclGetTbUtilization(rescclAlgo_t algo, char* json, size_t* len
   if (!a.opt.trace || !a.trace_host) fail(rescclInvalidUsage, "no trace: load with trace=1 (RESCCL_TRACE=1) and run");
   std::ostringstream o;
   o << "{\"lanes\":[";
-  double sum_idle = 0, max_idle = 0;
-  int n = 0;
+  double sum_idle = 0, max_idle = 0, csum = 0, cmax = 0;
+  int n = 0, nc = 0;
   unsigned long long t_min = ~0ull, t_max = 0;
   bool first = true;
   for (int b = 0; b < a.trace_blocks; ++b) {
@@ -1894,9 +1894,13 @@ rescclResult_t rescclGetTbUtilization(rescclAlgo_t algo, char* json, size_t* len
     int rank = 0;
     while (rank + 1 < (int)a.lay.pair_start.size() && a.lay.pair_start[rank + 1] <= pair) ++rank;
     int cta = pair - a.lay.pair_start[rank];
+    unsigned long long cb = ~0ull, ce = 0;
     for (int lane = 0; lane < 2; ++lane) {
-      volatile unsigned long long* tr = a.trace_host + 4 * (2 * (size_t)b + lane);
-      if (tr[3] == 0 || tr[1] <= tr[0]) continue;
+      volatile unsigned long long* tr = a.trace_host + 8 * (2 * (size_t)b + lane);
+      if (tr[1] <= tr[0]) continue;
+      cb = std::min(cb, (unsigned long long)tr[0]);
+      ce = std::max(ce, (unsigned long long)tr[1]);
+      if (tr[3] == 0) continue;
       double life = (double)(tr[1] - tr[0]);
       double idle = (double)tr[2] / life;
       if (idle > 1) idle = 1;
@@ -1909,11 +1913,20 @@ rescclResult_t rescclGetTbUtilization(rescclAlgo_t algo, char* json, size_t* len
         << "," << tr[2] << "," << tr[3] << "]";
       first = false;
     }
+    if (ce > cb) {  // the CTA (one SM): both lanes busy-waiting or finished
+      double ci = (double)a.trace_host[8 * (2 * (size_t)b) + 4] / (double)(ce - cb);
+      if (ci > 1) ci = 1;
+      csum += ci;
+      cmax = std::max(cmax, ci);
+      ++nc;
+    }
   }
-  double avg = n ? sum_idle / n : 0;
+  double avg = n ? sum_idle / n : 0, cavg = nc ? csum / nc : 0;
   o << "],\"fields\":[\"rank\",\"cta\",\"instance\",\"lane\",\"lifetime_ns\",\"wait_ns\",\"prims\"]"
     << ",\"tbs\":" << n << ",\"comm_time\":" << (1 - avg) << ",\"avg_idle\":" << avg
-    << ",\"max_idle\":" << max_idle << ",\"span_ns\":" << (n ? t_max - t_min : 0) << "}";
+    << ",\"max_idle\":" << max_idle << ",\"ctas\":" << nc << ",\"cta_comm_time\":" << (1 - cavg)
+    << ",\"cta_avg_idle\":" << cavg << ",\"cta_max_idle\":" << cmax
+    << ",\"span_ns\":" << (n ? t_max - t_min : 0) << "}";
   write_out(o.str(), json, len);
   API_END
 }

@@ -62,7 +62,7 @@ struct KArgs {
   int block_base;                     // global block id of blockIdx.x == 0
   int* err;                           // host-mapped error word
   u64 timeout_ns;
-  u64* trace;                         // RESCCL_TRACE: 4 x u64 per (block, lane), host-mapped
+  u64* trace;                         // RESCCL_TRACE: 8 x u64 per (block, lane), host-mapped
   u64 epoch;                          // RESCCL_EXIT_BARRIER: calls of this plan issued before
   u64* epochs;                        // device-side epochs (graph-capturable launches), or null:
                                       // {mb_base, epoch, CTAs done}; the kernel reads the first two
@@ -239,6 +239,14 @@ __device__ __forceinline__ u32 lds_u32(u32 a) {
 }
 __device__ __forceinline__ void sts_u32(u32 a, u32 v) {
   asm volatile("st.volatile.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ u64 lds_u64(u32 a) {
+  u64 v;
+  asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_u64(u32 a, u64 v) {
+  asm volatile("st.volatile.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
 }
 __device__ __forceinline__ u32 lds_u8(u32 a) {
   u32 v;
@@ -596,6 +604,7 @@ struct Lane {
   // gate = 1 + lane index of the last earlier same-lane primitive a dropped implied
   // dependency pointed at), the cursor (push receive wa_c, micro-batch wa_m) of the next
   // credit to post, the lane index of the running primitive and its push-receive index
+  u32 cta_idle;              // RESCCL_TRACE (smem): u32 lanes idle, u32 pad, u64 both-idle ns, u64 start[2]
   const PrimDesc* descs;
   const int* wa;
   const int* wg;
@@ -608,6 +617,9 @@ struct Lane {
   __device__ bool wait_ge(const u64* p, u64 target) {
     if (ready_ge(p, target)) return true;
     u64 t0 = globaltimer();
+#if RESCCL_TRACE
+    cta_idle_enter_(t0);
+#endif
     u32 spins = 0;
     while (!ready_ge(p, target)) {
 #if RESCCL_LOOKAHEAD
@@ -620,13 +632,65 @@ struct Lane {
       }
     }
 #if RESCCL_TRACE
-    wait_ns += globaltimer() - t0;
+    const u64 t1 = globaltimer();
+    wait_ns += t1 - t0;
+    cta_idle_exit_(t1);
 #endif
     return true;
   }
+  __device__ void cta_idle_enter_(u64 now);
+  __device__ void cta_idle_exit_(u64 now);
 };
 
 __device__ __forceinline__ u64* at(char* base, i64 off) { return (u64*)(base + off); }
+
+// RESCCL_TRACE: a lane leader's busy-waiting intervals (waiting for a peer's flag or
+// credit or for a local dependency, with no data of its own in flight).  Per lane they sum
+// to wait_ns (the paper's per-TB idle ratio, with a lane as the paper's TB);
+// per CTA the intervals in which BOTH lanes busy-wait (or have finished) are summed in
+// shared memory: the SM itself is then occupied without moving data.
+__device__ __forceinline__ void cta_idle_enter(const Lane& L, u64 now) {
+#if RESCCL_TRACE
+  sts_u64(L.cta_idle + 16 + 8 * (L.bar - 1), now);  // this lane's start, before the count
+  fence_cta();
+  asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(L.cta_idle) : "memory");
+#endif
+}
+__device__ __forceinline__ void cta_idle_exit(const Lane& L, u64 now) {
+#if RESCCL_TRACE
+  u32 old;
+  asm volatile("atom.shared.add.u32 %0, [%1], -1;" : "=r"(old) : "r"(L.cta_idle) : "memory");
+  if (old == 2) {  // both lanes were idle: from the later of the two starts until now
+    const u64 a0 = lds_u64(L.cta_idle + 16), a1 = lds_u64(L.cta_idle + 24);
+    const u64 st = a0 > a1 ? a0 : a1;
+    if (now > st) {
+      const u32 addr = L.cta_idle + 8;
+      const u64 d = now - st;
+      asm volatile("red.shared.add.u64 [%0], %1;" ::"r"(addr), "l"(d) : "memory");
+    }
+  }
+#endif
+}
+__device__ __forceinline__ void Lane::cta_idle_enter_(u64 now) { cta_idle_enter(*this, now); }
+__device__ __forceinline__ void Lane::cta_idle_exit_(u64 now) { cta_idle_exit(*this, now); }
+__device__ __forceinline__ void idle_on(Lane& L, u64& t_idle) {
+#if RESCCL_TRACE
+  if (t_idle == 0) {
+    t_idle = globaltimer();
+    cta_idle_enter(L, t_idle);
+  }
+#endif
+}
+__device__ __forceinline__ void idle_off(Lane& L, u64& t_idle) {
+#if RESCCL_TRACE
+  if (t_idle) {
+    const u64 now = globaltimer();
+    L.wait_ns += now - t_idle;
+    cta_idle_exit(L, now);
+  }
+#endif
+  t_idle = 0;
+}
 
 // RESCCL_PHASE record (leader only): kind 0 = blocking register path, 1 = flag-only
 // primitive, 2 = TMA lane engine; t[0..4] as documented at each call site.
@@ -988,14 +1052,6 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
 // parity of a quiescent mbarrier's current (incomplete) phase: the preceding phase, of
 // the other parity, tests complete
 __device__ __forceinline__ u32 mbar_phase(u32 bar) { return mbar_test(bar, 0) ? 1u : 0u; }
-__device__ __forceinline__ u64 lds_u64(u32 a) {
-  u64 v;
-  asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
-  return v;
-}
-__device__ __forceinline__ void sts_u64(u32 a, u64 v) {
-  asm volatile("st.volatile.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
-}
 // i-th (0-based) set bit of m
 __device__ __forceinline__ u32 nth_bit(u32 m, u32 i) {
   for (; i; --i) m &= m - 1;
@@ -1096,7 +1152,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   lo_p = lo_l;
   nb_p = nb_l;
   u32 gp_end = T_l;           // tiles through micro-batch pj
-  u64 t_idle = 0;
+  u64 t_idle = 0, t_wd = 0;  // idle interval start (trace), watchdog start
   u32 spins = 0;
   const u64 pol_first = policy_evict_first();
   const u64 pol_last = policy_evict_last();
@@ -1350,15 +1406,13 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
     }
 #endif
     if (prog) {
-#if RESCCL_TRACE
-      if (t_idle) L.wait_ns += globaltimer() - t_idle;
-#endif
+      idle_off(L, t_idle);
       spins = 0;
-      t_idle = 0;
     } else {
-#if RESCCL_TRACE
-      if (t_idle == 0) t_idle = globaltimer();
-#endif
+      // idle = busy-waiting with no data of this lane in flight (tiles outstanding are the
+      // data path working, not a wait for a peer)
+      if (stored == issued) idle_on(L, t_idle);
+      else idle_off(L, t_idle);
 #if RESCCL_LOOKAHEAD
       if (L.wa_c < L.wa_n && stored == issued && (spins & 3) == 0) lookahead(L);  // only while data-idle
 #endif
@@ -1375,14 +1429,15 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       }
       if ((spins & 255) == 0) {
         const u64 now = globaltimer();
-        if (t_idle == 0) t_idle = now;
-        else if (now - t_idle > a.timeout_ns) {
+        if (t_wd == 0) t_wd = now;
+        else if (now - t_wd > a.timeout_ns) {
           atomicCAS(a.err, 0, kErrTimeout);
           *L.abort_flag = 1;
           return false;
         }
       }
     }
+    if (prog) t_wd = 0;
   }
   if (stored > released) {  // (all posted: every store has completed)
     tma_wait_read_n(0);
@@ -1393,9 +1448,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   if (wanting) sts_u32(want_self, 0u);
 #endif
 #undef RESCCL_HS
-#if RESCCL_TRACE
-  if (t_idle) L.wait_ns += globaltimer() - t_idle;
-#endif
+  idle_off(L, t_idle);
   L.tseq = k0 + issued;
   L.cpar = Lcpar;
   return true;
@@ -1504,7 +1557,7 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
   const u64 mb_base = a.mb_base;
   constexpr bool recv = F & kRecv;
   int wp = 0, dj = 0;  // posted (readable / writable) / completed micro-batches
-  u64 t_idle = 0;
+  u64 t_idle = 0, t_wd = 0;  // idle interval start (trace), watchdog start
   u32 spins = 0;
   // phase records: t0 start of the wait, t1 dependencies met (readable / writable
   // posted right after), t2 the peer's "written" flag seen (push receive), t4 posted
@@ -1559,23 +1612,19 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
       }
     }
     if (prog) {
-#if RESCCL_TRACE
-      if (t_idle) L.wait_ns += globaltimer() - t_idle;
-#endif
+      idle_off(L, t_idle);
       spins = 0;
-      t_idle = 0;
+      t_wd = 0;
     } else {
-#if RESCCL_TRACE
-      if (t_idle == 0) t_idle = globaltimer();
-#endif
+      idle_on(L, t_idle);
 #if RESCCL_LOOKAHEAD
       if (L.wa_c < L.wa_n && (spins & 7) == 7) lookahead(L);  // rate-limited: the flag poll first
 #endif
       if (++spins > 32) nanosleep_(20);
       if ((spins & 255) == 0) {
         const u64 now = globaltimer();
-        if (t_idle == 0) t_idle = now;
-        else if (now - t_idle > a.timeout_ns) {
+        if (t_wd == 0) t_wd = now;
+        else if (now - t_wd > a.timeout_ns) {
           atomicCAS(a.err, 0, kErrTimeout);
           *L.abort_flag = 1;
           return false;
@@ -1583,9 +1632,7 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
       }
     }
   }
-#if RESCCL_TRACE
-  if (t_idle) L.wait_ns += globaltimer() - t_idle;
-#endif
+  idle_off(L, t_idle);
   return true;
 }
 

@@ -99,3 +99,41 @@ def test_fig16_program_text_on_gpu(dtype):
     _check(outs, exp)
     if dtype == "int32":
         _check(outs, definition.allreduce(xs, "int32"))
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("name,coll,kw", [("ring", "allreduce", {}), ("hm", "allreduce", {"g": 4}),
+                                          ("dbt", "allreduce", {})])
+def test_tb_utilization_trace(name, coll, kw):
+    """Table 3 instrumentation (trace=1): per-lane (the paper's TB)
+    and per-CTA idle ratios are well-formed, one lane record per traced lane, and tracing
+    leaves the result bit-exact."""
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    n = 8
+    g = oir.generate(name, coll, n, **kw)
+    count = (1 << 20) + 333
+    for k, v in dict(chunkbytes=1 << 18, instances=2, fifodepth=2, direct=1, trace=1, nwarps=8).items():
+        g.extra[k] = str(v)
+    xs = inp.all_inputs("float32", 24, n, count)
+    grp = R.VirtualGroup(n, 0)
+    try:
+        import torch
+        from gpu_helpers import to_numpy, to_torch
+        grp.load(g.to_text())
+        info = grp.plan_info()
+        s = [to_torch(x, "float32") for x in xs]
+        r = [torch.empty_like(t) for t in s]
+        grp.allreduce(s, r)
+        torch.cuda.synchronize()
+        assert grp.async_error() == 0
+        u = R.rescclGetTbUtilization(grp.comms[0].algos[-1])
+        outs = [to_numpy(t, "float32") for t in r]
+    finally:
+        grp.destroy()
+    lanes = sum(len(a) > 0 for rk in info["plan"]["ranks"] for c in rk["ctas"] for a in (c["send"], c["recv"]))
+    assert u["tbs"] == lanes * info["instances"]
+    assert u["ctas"] == sum(info["blocks_per_rank"])
+    for k in ("comm_time", "avg_idle", "max_idle", "cta_comm_time", "cta_avg_idle", "cta_max_idle"):
+        assert 0.0 <= u[k] <= 1.0, (k, u[k])
+    exp = replay.replay(lower.lower(g, direct=True), xs, "float32", count, chunk_bytes=1 << 18, instances=2, K=2)
+    _check(outs, exp)

@@ -53,7 +53,10 @@ for name, coll, gopts, popts in cases:
            "paper_tbs_per_rank": paper_tbs, "n_connections": [rk["n_connections"] for rk in info["plan"]["ranks"]],
            "instances": info["instances"], "traced_lanes": u["tbs"], "comm_time": round(u["comm_time"], 4),
            "avg_idle": round(u["avg_idle"], 4), "max_idle": round(u["max_idle"], 4),
-           "span_us": round(u["span_ns"] / 1e3, 1), "fused": info["plan"]["fused"]}
+           "span_us": round(u["span_ns"] / 1e3, 1), "fused": info["plan"]["fused"],
+           # per CTA (= one SM): fraction of its lifetime with both lanes busy-waiting / done
+           "ctas": u["ctas"], "cta_comm_time": round(u["cta_comm_time"], 4),
+           "cta_avg_idle": round(u["cta_avg_idle"], 4), "cta_max_idle": round(u["cta_max_idle"], 4)}
     out.append(row)
     print(json.dumps(row), flush=True)
     grp.destroy()
