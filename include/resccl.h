@@ -36,7 +36,18 @@
  *    device sendbuf runs as one piece.  The host in-place rules are the device ones.
  *    Host-buffer calls refuse CUDA-graph capture (InvalidUsage).  Staged calls of a
  *    direct=1 algorithm across processes run its staged twin (the stage is not a
- *    registered window).
+ *    registered window).  The piece size is read once when a communicator is created;
+ *    multi-process ranks must agree on it (rescclCommConnect: InvalidUsage otherwise).
+ *    Every rank of a call must use the same placement (all host or all device buffers,
+ *    per send / receive side): the placement decides the piece schedule and transport,
+ *    i.e. the launches every rank must issue alike; mixed placement across processes is
+ *    undefined (it hangs until the watchdog fires).  Single-process multi-device
+ *    communicators refuse pageable host buffers (InvalidArgument: one host thread drives
+ *    every rank, and a pageable download would block it on ranks not yet issued).  A
+ *    pointer the runtime cannot classify is InvalidArgument.
+ *  - ReduceScatter uses communicator-owned scratch that grows with the largest call;
+ *    growing inside a CUDA-graph capture is refused (InvalidUsage): run one call of the
+ *    largest size eagerly first.
  *  - All ranks issue the same collectives in the same order with the same count,
  *    dtype and op; a communicator is not thread-safe.
  *  - Every function returns a rescclResult_t; no exception crosses the ABI and the

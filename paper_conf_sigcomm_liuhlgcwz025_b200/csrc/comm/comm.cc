@@ -429,6 +429,11 @@ struct rescclComm {
   char* hstage = nullptr;
   size_t hstage_bytes = 0;
   HostCopy hcopy;  // host-buffer collectives: copy streams (multi-process / multi-device)
+  // host-buffer piece size (RESCCL_HOST_PIECE), fixed at creation; multi-process ranks
+  // check at connect that every rank uses the same value (the piece schedule decides the
+  // launches every rank must issue alike)
+  size_t host_piece = 0;
+  std::vector<char*> retired_scratch;  // scratch buffers replaced by larger ones (freed at destroy)
 };
 
 namespace {
@@ -640,16 +645,19 @@ Geometry call_geometry(const AlgoShared& a, const CallDesc& c) {
   return geometry(a.ir.coll, a.ir.nranks, (int64_t)c.count, elt_size(c.dt), a.opt.chunk_bytes, a.opt.instances);
 }
 
-void ensure_scratch(rescclComm* comm, size_t bytes) {
+void ensure_scratch(rescclComm* comm, size_t bytes, cudaStream_t s = nullptr) {
   if (comm->scratch_bytes >= bytes) return;
+  // growing allocates: not allowed inside a CUDA-graph capture (the capture would be
+  // invalidated) -- the first ReduceScatter of a size must run eagerly before capturing
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (s && cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone)
+    fail(rescclInvalidUsage, "ReduceScatter scratch would grow during CUDA-graph capture: run one call of this "
+                             "size (or larger) eagerly before capturing");
   cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
   char* p = nullptr;
   cuda_check(cudaMalloc((void**)&p, bytes), "cudaMalloc(scratch)");
-  // the old buffer may still be in use by queued kernels: keep it until destroy
-  if (comm->scratch) {
-    static std::vector<char*> graveyard;
-    graveyard.push_back(comm->scratch);
-  }
+  // the old buffer may still be in use by queued kernels: keep it until rescclCommDestroy
+  if (comm->scratch) comm->retired_scratch.push_back(comm->scratch);
   comm->scratch = p;
   comm->scratch_bytes = bytes;
 }
@@ -746,7 +754,7 @@ void launch_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const vo
     }
   }
   if (a.ir.coll == Coll::ReduceScatter) {
-    ensure_scratch(comm, c.count * comm->nranks * elt_size(c.dt));
+    ensure_scratch(comm, c.count * comm->nranks * elt_size(c.dt), s);
     ka.scratch[comm->rank] = comm->scratch;
   }
   fill_geometry(ka, g, c.count);
@@ -778,7 +786,7 @@ void group_launch(Group* G, Pending& p) {
     ka.sendbuf[q] = (const char*)p.send[q];
     ka.recvbuf[q] = (char*)p.recv[q];
     if (a.ir.coll == Coll::ReduceScatter) {
-      ensure_scratch(G->comms[q], c.count * G->nranks * elt_size(c.dt));
+      ensure_scratch(G->comms[q], c.count * G->nranks * elt_size(c.dt), p.streams.back());
       ka.scratch[q] = G->comms[q]->scratch;
     }
   }
@@ -825,12 +833,16 @@ void group_launch(Group* G, Pending& p) {
 // full duplex).  The
 // caller's stream waits for the last download: stream semantics are the device path's.
 
-bool host_ptr(const void* p) {
+// Host (pinned or pageable) vs device memory.  A pointer the runtime cannot classify is
+// an error (InvalidArgument), never silently treated as host memory.
+bool host_ptr(const void* p, bool* pageable = nullptr) {
   cudaPointerAttributes at;
-  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+  cudaError_t e = cudaPointerGetAttributes(&at, p);
+  if (e != cudaSuccess) {
     cudaGetLastError();
-    return true;
+    fail(rescclInvalidArgument, std::string("buffer pointer not classifiable: ") + cudaGetErrorString(e));
   }
+  if (pageable) *pageable = at.type == cudaMemoryTypeUnregistered;
   return at.type == cudaMemoryTypeHost || at.type == cudaMemoryTypeUnregistered;
 }
 
@@ -931,7 +943,10 @@ struct Staging {
   }
 };
 
-size_t piece_elems(size_t count, size_t e) { return std::min(count, std::max<size_t>(1, host_piece_bytes() / e)); }
+size_t piece_elems(const rescclComm* comm, size_t count, size_t e) {
+  const size_t pb = comm->host_piece ? comm->host_piece : host_piece_bytes();
+  return std::min(count, std::max<size_t>(1, pb / e));
+}
 
 // multi-process / multi-device rank
 void host_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const void* send, void* recv,
@@ -941,7 +956,7 @@ void host_rank(rescclComm* comm, rescclAlgo* algo, const CallDesc& c, const void
   P.plan(c.coll, comm->rank, comm->nranks, send, recv, c.count, e);
   ensure_hstage(comm, P.need);
   P.stage = comm->hstage;
-  const size_t pe = P.pieces ? piece_elems(c.count, e) : c.count, np = (c.count + pe - 1) / pe;
+  const size_t pe = P.pieces ? piece_elems(comm, c.count, e) : c.count, np = (c.count + pe - 1) / pe;
   HostCopy& h = comm->hcopy;
   ensure_copy(h, 2 * np + 2);
   size_t ei = 0;
@@ -983,7 +998,7 @@ void group_host_launch(Group* G, Pending& p) {
     any_hr |= P[q].hr;
     pieces &= P[q].pieces;
   }
-  const size_t pe = pieces ? piece_elems(p.count, e) : p.count, np = (p.count + pe - 1) / pe;
+  const size_t pe = pieces ? piece_elems(G->comms[0], p.count, e) : p.count, np = (p.count + pe - 1) / pe;
   cudaStream_t ls = p.streams.back();
   std::vector<cudaStream_t> others;
   for (auto s : p.streams)
@@ -1050,7 +1065,14 @@ void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t
   const bool capturing = cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone;
   if (capturing && !comm->active[coll])
     fail(rescclInvalidUsage, "load an algorithm before capturing a collective into a CUDA graph");
-  const bool host = count > 0 && (host_ptr(send) || host_ptr(recv));
+  bool pg_send = false, pg_recv = false;
+  const bool host = count > 0 && (host_ptr(send, &pg_send) | host_ptr(recv, &pg_recv));
+  // one host thread drives every rank of a single-process multi-device communicator: a
+  // pageable download blocks that thread until this rank's collective finishes, which
+  // waits for ranks the thread has not issued yet -- refuse instead of hanging
+  if (comm->mode == 2 && (pg_send || pg_recv))
+    fail(rescclInvalidArgument, "pageable host buffers are not supported with single-process multi-device "
+                                "communicators (pin them, e.g. cudaHostRegister / tensor.pin_memory())");
   if (capturing && host)
     fail(rescclInvalidUsage, "host buffers cannot be captured into a CUDA graph (staged copies)");
   rescclAlgo* algo = ensure_algo(comm, (Coll)coll);
@@ -1499,6 +1521,7 @@ struct Blob {
   unsigned long long arena_bytes;
   cudaIpcMemHandle_t handle;
   int pid;
+  unsigned long long host_piece;  // RESCCL_HOST_PIECE of this rank (must agree across ranks)
 };
 
 rescclResult_t rescclCommCreate(int rank, int nranks, int cudaDev, rescclComm_t* out) {
@@ -1512,6 +1535,7 @@ rescclResult_t rescclCommCreate(int rank, int nranks, int cudaDev, rescclComm_t*
   c->mode = 0;
   cuda_check(cudaSetDevice(cudaDev), "cudaSetDevice");
   c->arena_bytes = arena_default();
+  c->host_piece = host_piece_bytes();
   cuda_check(cudaMalloc((void**)&c->arena, c->arena_bytes), "cudaMalloc(arena)");
   cuda_check(cudaMemset(c->arena, 0, c->arena_bytes), "cudaMemset(arena)");
   cuda_check(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
@@ -1540,6 +1564,7 @@ rescclResult_t rescclCommGetHandle(rescclComm_t comm, void* buf, size_t* len) {
   b.dev = comm->dev;
   b.arena_bytes = comm->arena_bytes;
   b.pid = (int)getpid();
+  b.host_piece = comm->host_piece;
   cuda_check(cudaSetDevice(comm->dev), "cudaSetDevice");
   cuda_check(cudaIpcGetMemHandle(&b.handle, comm->arena), "cudaIpcGetMemHandle");
   memcpy(buf, &b, sizeof(b));
@@ -1560,6 +1585,9 @@ rescclResult_t rescclCommConnect(rescclComm_t comm, const void* const* handles, 
     if (b.magic != 0x52435343u || b.rank != q || b.nranks != comm->nranks)
       fail(rescclInvalidArgument, "handle blob of rank " + std::to_string(q) + " is inconsistent");
     if (b.arena_bytes != comm->arena_bytes) fail(rescclInvalidUsage, "ranks use different RESCCL_ARENA_BYTES");
+    if (b.host_piece != comm->host_piece)
+      fail(rescclInvalidUsage, "ranks use different RESCCL_HOST_PIECE (" + std::to_string(b.host_piece) + " on rank " +
+                                   std::to_string(q) + ", " + std::to_string(comm->host_piece) + " here)");
     void* p = nullptr;
     cudaError_t e = cudaIpcOpenMemHandle(&p, b.handle, cudaIpcMemLazyEnablePeerAccess);
     if (e != cudaSuccess)
@@ -1698,6 +1726,7 @@ rescclResult_t rescclCommInitAll(rescclComm_t* comms, int ndev, const int* devli
       c->nranks = ndev;
       c->dev = devs[0];
       c->mode = 1;
+      c->host_piece = host_piece_bytes();
       c->group = G;
       c->connected = true;
       c->err_host = G->err_host;
@@ -1714,6 +1743,7 @@ rescclResult_t rescclCommInitAll(rescclComm_t* comms, int ndev, const int* devli
       c->nranks = ndev;
       c->dev = devs[r];
       c->mode = 2;
+      c->host_piece = host_piece_bytes();
       cuda_check(cudaSetDevice(devs[r]), "cudaSetDevice");
       for (int q = 0; q < ndev; ++q) {
         if (q == r) continue;
@@ -1768,6 +1798,7 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
     }
     // this rank's buffers (the group's other comms may already be deleted)
     if (comm->scratch) cudaFree(comm->scratch);
+    for (char* q : comm->retired_scratch) cudaFree(q);
     if (comm->hstage) cudaFree(comm->hstage);
   } else {
     for (auto& a : comm->algos) {
@@ -1788,6 +1819,7 @@ rescclResult_t rescclCommDestroy(rescclComm_t comm) {
     if (comm->arena) cudaFree(comm->arena);
     if (comm->err_host) cudaFreeHost(comm->err_host);
     if (comm->scratch) cudaFree(comm->scratch);
+    for (char* q : comm->retired_scratch) cudaFree(q);
     if (comm->hstage) cudaFree(comm->hstage);
     comm->hcopy.release();
   }
