@@ -83,6 +83,7 @@ struct Driver {
   CUresult (*GetErrorString)(CUresult, const char**) = nullptr;
   CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
   CUresult (*MemGetAddressRange)(CUdeviceptr*, size_t*, CUdeviceptr) = nullptr;
+  CUresult (*OccupancyMaxActiveBlocksPerMultiprocessor)(int*, CUfunction, int, size_t) = nullptr;
   bool ok = false;
 };
 
@@ -108,6 +109,7 @@ Driver& driver() {
       entry("cuGetErrorString", &d.GetErrorString);
       entry("cuFuncSetAttribute", &d.FuncSetAttribute);
       entry("cuMemGetAddressRange", &d.MemGetAddressRange);
+      entry("cuOccupancyMaxActiveBlocksPerMultiprocessor", &d.OccupancyMaxActiveBlocksPerMultiprocessor);
       d.ok = true;
     } catch (Error&) {
       d.ok = false;
@@ -346,6 +348,8 @@ struct Kern {
   CUmodule mod = nullptr;
   CUfunction fn = nullptr;
   int smem = 0;
+  int max_grid = -1;  // co-resident blocks (cooperative launch limit), per block size
+  int max_grid_block = 0;
 };
 
 struct AlgoShared {
@@ -663,6 +667,21 @@ void ensure_scratch(rescclComm* comm, size_t bytes, cudaStream_t s = nullptr) {
 }
 
 void launch(Kern& k, int grid, int block, KArgs& args, cudaStream_t s) {
+  // every CTA of a schedule must be co-resident (they wait on each other): check before
+  // the cooperative launch so the error names the cause
+  if (k.max_grid < 0 || k.max_grid_block != block) {
+    int per_sm = 0, dev = 0, nsm = 0;
+    cu_check(driver().OccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k.fn, block, (size_t)k.smem),
+             "cuOccupancyMaxActiveBlocksPerMultiprocessor");
+    cuda_check(cudaGetDevice(&dev), "cudaGetDevice");
+    cuda_check(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev), "cudaDeviceGetAttribute");
+    k.max_grid = per_sm * nsm;
+    k.max_grid_block = block;
+  }
+  if (grid > k.max_grid)
+    fail(rescclInvalidUsage, "the plan needs " + std::to_string(grid) + " co-resident CTAs (CTAs per rank x "
+                             "instances x ranks on this device) but at most " + std::to_string(k.max_grid) +
+                             " fit: lower instances / nwarps / the TB budget");
   void* params[] = {&args};
   cu_check(driver().LaunchCooperativeKernel(k.fn, grid, 1, 1, block, 1, 1, k.smem, (CUstream)s, params),
            "cuLaunchCooperativeKernel");

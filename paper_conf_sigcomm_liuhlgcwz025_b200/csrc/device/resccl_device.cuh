@@ -70,6 +70,13 @@ struct KArgs {
   u64* phase;                         // RESCCL_PHASE: RESCCL_PH_MAX x 8 u64 per (block, lane), or null
 };
 
+// CTA barrier that tolerates warp divergence (barrier.sync without .aligned): a lane's
+// leader thread runs leader-only primitives (flag loops) while the rest of its warp has
+// already moved on, so the block-wide barriers after the lanes' lists and the lane
+// barriers may be reached by a warp's threads at different times (__syncthreads is the
+// .aligned form, undefined under divergence; compute-sanitizer synccheck flags it)
+__device__ __forceinline__ void cta_sync() { asm volatile("barrier.sync 0;" ::: "memory"); }
+
 // Device-side epochs: every CTA takes this launch's micro-batch base and call epoch from
 // device memory (so a CUDA graph replays with fresh epochs); the last CTA to finish
 // advances them by this call's micro-batches / one call.  Stream order makes the update
@@ -81,12 +88,12 @@ __device__ __forceinline__ const KArgs* epochs_begin(const KArgs& a, KArgs* sh) 
     sh->mb_base = *(volatile u64*)&a.epochs[0];
     sh->epoch = *(volatile u64*)&a.epochs[1];
   }
-  __syncthreads();
+  cta_sync();
   return sh;
 }
 __device__ __forceinline__ void epochs_end(const KArgs& a) {
   if (!a.epochs) return;
-  __syncthreads();
+  cta_sync();
   if (threadIdx.x != 0) return;
   __threadfence();
   const unsigned long long old = atomicAdd((unsigned long long*)&a.epochs[2], 1ull);
@@ -611,7 +618,7 @@ struct Lane {
   int wa_n, wa_c, wa_m, lpos, wai;
 
   __device__ __forceinline__ void sync() const {
-    asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(nthreads) : "memory");
+    asm volatile("barrier.sync %0, %1;" ::"r"(bar), "r"(nthreads) : "memory");  // (divergence-tolerant)
   }
   // leader only: spin until *p >= target; false on timeout (error word set)
   __device__ bool wait_ge(const u64* p, u64 target) {
@@ -1502,7 +1509,7 @@ __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const Prim
           if ((spins & 1023) == 0 && *abort_flag) break;
         }
       }
-      asm volatile("bar.sync %0, %1;" ::"r"(Lbar + 2), "r"(nct) : "memory");
+      asm volatile("barrier.sync %0, %1;" ::"r"(Lbar + 2), "r"(nct) : "memory");
       if (*abort_flag) return false;
       w = lds_u64(Lqprog);
 #else
@@ -1706,7 +1713,7 @@ __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
 // block adds 1 to its rank's monotone done counter (release); block 0 then waits until
 // each peer's counter covers this call: (epoch + 1) x that peer's block count.
 __device__ __noinline__ void exit_barrier(const KArgs& a, int rank, int nranks, const int* blocks, i64 off) {
-  __syncthreads();
+  cta_sync();
   if (threadIdx.x != 0) return;
   fence_release();
   asm volatile("red.release" RESCCL_SC ".global.add.u64 [%0], 1;" ::"l"(at(a.arena[rank], off)) : "memory");

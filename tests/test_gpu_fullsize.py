@@ -80,7 +80,7 @@ def test_fullsize_elementwise(inplace):
     ("dbt", "allreduce", {}, 64, "float16", dict(instances=4, chunkbytes=1 << 20, fifodepth=2)),
     # C4: synthesized AllGather / ReduceScatter (total buffer sizes)
     ("synth", "reducescatter", {"seed": 0, "fanout": 2}, 256, "float32", dict(instances=4, chunkbytes=1 << 20)),
-    ("synth", "allgather", {"seed": 1, "fanout": 3}, 256, "bfloat16", dict(instances=4, chunkbytes=4 << 20, direct=1)),
+    ("synth", "allgather", {"seed": 1, "fanout": 3}, 256, "bfloat16", dict(instances=3, chunkbytes=4 << 20, direct=1)),
 ])
 def test_fullsize_fast(name, coll, gkw, size_mb, dtype, opts):
     import torch
