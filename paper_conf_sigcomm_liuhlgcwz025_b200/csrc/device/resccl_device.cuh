@@ -78,32 +78,33 @@ struct KArgs {
 __device__ __forceinline__ void cta_sync() { asm volatile("barrier.sync 0;" ::: "memory"); }
 
 // Device-side epochs: every CTA takes this launch's micro-batch base and call epoch from
-// device memory (so a CUDA graph replays with fresh epochs); the last CTA to finish
-// advances them by this call's micro-batches / one call.  Stream order makes the update
-// visible to the next launch of the plan.
+// device memory (so a CUDA graph replays with fresh epochs).  Each CTA reads them with
+// acquire loads (its arrival below cannot overtake the reads) and then counts itself in;
+// the LAST CTA to arrive -- every CTA of this launch has read the old values by then --
+// advances them by this call's micro-batches / one call and resets the count, right at
+// the start of the kernel, off its critical path (r02: the former end-of-kernel fence +
+// atomic cost every launch ~1-2 us of tail).  Stream order makes the update visible to
+// the next launch of the plan.
 __device__ __forceinline__ const KArgs* epochs_begin(const KArgs& a, KArgs* sh) {
   if (!a.epochs) return &a;
   if (threadIdx.x == 0) {
     *sh = a;
-    sh->mb_base = *(volatile u64*)&a.epochs[0];
-    sh->epoch = *(volatile u64*)&a.epochs[1];
+    u64 mb, ep;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(mb) : "l"(&a.epochs[0]) : "memory");
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(ep) : "l"(&a.epochs[1]) : "memory");
+    sh->mb_base = mb;
+    sh->epoch = ep;
+    const unsigned long long old = atomicAdd((unsigned long long*)&a.epochs[2], 1ull);
+    if (old == (unsigned long long)gridDim.x - 1) {
+      a.epochs[0] = mb + (u64)a.n_mb;
+      a.epochs[1] = ep + 1;
+      a.epochs[2] = 0;
+    }
   }
   cta_sync();
   return sh;
 }
-__device__ __forceinline__ void epochs_end(const KArgs& a) {
-  if (!a.epochs) return;
-  cta_sync();
-  if (threadIdx.x != 0) return;
-  __threadfence();
-  const unsigned long long old = atomicAdd((unsigned long long*)&a.epochs[2], 1ull);
-  if (old == (unsigned long long)gridDim.x - 1) {
-    a.epochs[0] += (u64)a.n_mb;
-    a.epochs[1] += 1;
-    a.epochs[2] = 0;
-    __threadfence();
-  }
-}
+__device__ __forceinline__ void epochs_end(const KArgs&) {}
 
 enum : int { kRecv = 1, kSend = 2, kReduce = 4, kStore = 8, kCopy = 16, kDirect = 32, kPull = 64, kSendPull = 128 };
 enum : int { BufNone = -1, BufSend = 0, BufRecv = 1, BufScratch = 2 };

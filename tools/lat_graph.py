@@ -15,6 +15,7 @@ import paper_conf_sigcomm_liuhlgcwz025_b200 as R  # noqa: E402
 
 N, REPS = int(os.environ.get("LAT_N", "8")), 20
 ALGO = os.environ.get("LAT_ALGO", "ring")
+GOPTS = os.environ.get("LAT_GOPTS", "g=4" if ALGO == "hm" else "")
 OPTS = sys.argv[1:] or ["instances=14 nwarps=8 chunkbytes=33554432 fifodepth=2 direct=1"]
 SIZES = [int(x) for x in os.environ.get("LAT_SIZES", "[1024, 65536, 1048576, 16777216, 67108864]")[1:-1].split(",")]
 
@@ -45,7 +46,7 @@ def main():
     print(json.dumps({"reference": "empty torch kernel in a graph", "us": round(graph_time(lambda: x.add_(1), st), 2)}),
           flush=True)
     for opts in OPTS:
-        text = R.rescclGenerateIr(ALGO, "allreduce", N, "g=4" if ALGO == "hm" else "")
+        text = R.rescclGenerateIr(ALGO, "allreduce", N, GOPTS)
         h, rest = text.split("\n", 1)
         grp = R.VirtualGroup(N, 0)
         grp.load(h + " " + opts + "\n" + rest)
@@ -58,7 +59,7 @@ def main():
             torch.cuda.synchronize()
             us = graph_time(lambda: grp.allreduce(s, r, stream=st), st)
             bus = S / (us * 1e-6) / 1e9 * 2 * (N - 1) / N
-            print(json.dumps({"opts": opts, "algo": ALGO, "bytes": S, "graph_us": round(us, 2),
+            print(json.dumps({"opts": opts, "algo": ALGO, "gopts": GOPTS, "bytes": S, "graph_us": round(us, 2),
                               "busbw_gbs": round(bus, 2), "err": grp.async_error()}), flush=True)
             del s, r
         grp.destroy()
