@@ -167,12 +167,18 @@ rescclResult_t rescclCommGetAsyncError(rescclComm_t comm, rescclResult_t* err);
  * Environment overrides: RESCCL_INSTANCES, RESCCL_CHUNK_BYTES, RESCCL_FIFO_DEPTH,
  * RESCCL_NWARPS, RESCCL_LINK_MODEL, RESCCL_FUSE, RESCCL_TB_BUDGET.
  * The loaded algorithm becomes the active one for its collective; with none
- * loaded, the built-in ring is used.  All ranks must load the same algorithms in
- * the same order.  InvalidUsage: nranks != communicator size, invalid IR (I6),
- * same-step conflicts, deadlocking plan. */
+ * loaded, the built-in ring is used.  Size-based selection: header options
+ * [minbytes=a] [maxbytes=b] give the range of per-rank buffer sizes S (AllReduce
+ * count x elt; AllGather / ReduceScatter N x count x elt) an algorithm serves; a call
+ * runs the most recently loaded or activated algorithm of its collective whose range
+ * holds its S (default range: every size), so e.g. a full-mesh schedule can serve small
+ * messages and a ring large ones.  All ranks must load the same algorithms in the same
+ * order.  InvalidUsage: nranks != communicator size, invalid IR (I6), same-step
+ * conflicts, deadlocking plan. */
 rescclResult_t rescclLoadAlgorithm(rescclComm_t comm, const char* irText, rescclAlgo_t* out);
 
-/* Make a previously loaded algorithm the active one for its collective. */
+/* Make a previously loaded algorithm the active one for its collective (and the most
+ * recent one for size-based selection). */
 rescclResult_t rescclSetActiveAlgorithm(rescclComm_t comm, rescclAlgo_t algo);
 
 /* JSON description of the lowered plan (Pr, per-rank CTAs/lanes/primitives,

@@ -162,6 +162,11 @@ struct Options {
   int sys_rank = -1; // rescclCompileIr / rescclCodegenIr: one rank's multi-process (.sys) kernel
   int nvls = 0;      // f3: NVLS transport for calls whose buffers lie in NVLS windows
   int nvls_ctas = 16;  // CTAs (x 512 threads) per rank of an NVLS launch
+  // size range this algorithm serves (bytes of the per-rank buffer S: AR count x elt, AG /
+  // RS N x count x elt); a call picks the most recently loaded / activated algorithm of its
+  // collective whose range holds its size (a size-based tuner over loaded schedules)
+  long long min_bytes = 0;
+  long long max_bytes = -1;  // -1: unbounded
 };
 
 std::map<std::string, std::string> parse_kv(const char* s) {
@@ -218,6 +223,8 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "devepoch") o.devepoch = (int)to_long(v, k);
   else if (k == "nvls") o.nvls = (int)to_long(v, k);
   else if (k == "nvlsctas") o.nvls_ctas = (int)to_long(v, k);
+  else if (k == "minbytes") o.min_bytes = to_long(v, k);
+  else if (k == "maxbytes") o.max_bytes = to_long(v, k);
   else if (k == "sched") {
     if (v == "hpds") o.sched = 0;
     else if (v == "rr") o.sched = 1;
@@ -416,6 +423,7 @@ struct rescclComm {
   int* err_dev = nullptr;
   std::vector<std::unique_ptr<rescclAlgo>> algos;
   rescclAlgo* active[3] = {nullptr, nullptr, nullptr};
+  std::vector<rescclAlgo*> ranked[3];  // per collective, activation order (most recent last)
   char* scratch = nullptr;
   size_t scratch_bytes = 0;
   std::vector<rescclComm*> peers_local;  // mode 2: every comm of the process
@@ -683,8 +691,20 @@ void launch(Kern& k, int grid, int block, KArgs& args, cudaStream_t s) {
                              "instances x ranks on this device) but at most " + std::to_string(k.max_grid) +
                              " fit: lower instances / nwarps / the TB budget");
   void* params[] = {&args};
-  cu_check(driver().LaunchCooperativeKernel(k.fn, grid, 1, 1, block, 1, 1, k.smem, (CUstream)s, params),
-           "cuLaunchCooperativeKernel");
+  // cooperative launch: the driver schedules the grid only when every CTA can be resident
+  // (a plain launch could start part of the grid beside a concurrent compute kernel, whose
+  // CTAs would then wait on CTAs not yet running).  RESCCL_COOP=0 (measurement aid) uses a
+  // plain launch.
+  static const bool coop = [] {
+    const char* v = getenv("RESCCL_COOP");
+    return !(v && v[0] == '0');
+  }();
+  if (coop)
+    cu_check(driver().LaunchCooperativeKernel(k.fn, grid, 1, 1, block, 1, 1, k.smem, (CUstream)s, params),
+             "cuLaunchCooperativeKernel");
+  else
+    cu_check(driver().LaunchKernel(k.fn, grid, 1, 1, block, 1, 1, k.smem, (CUstream)s, params, nullptr),
+             "cuLaunchKernel");
 }
 
 void fill_geometry(KArgs& ka, const Geometry& g, size_t count) {
@@ -1065,6 +1085,7 @@ void group_host_launch(Group* G, Pending& p) {
 }
 
 rescclAlgo* ensure_algo(rescclComm* comm, Coll coll);
+rescclAlgo* select_algo(rescclComm* comm, Coll coll, long long bytes);
 bool try_nvls(rescclComm* comm, const AlgoShared& a, int coll, const void* send, void* recv, size_t count,
               rescclDataType_t dt, rescclRedOp_t op, cudaStream_t s);
 
@@ -1094,7 +1115,8 @@ void collective(rescclComm* comm, int coll, const void* send, void* recv, size_t
                                 "communicators (pin them, e.g. cudaHostRegister / tensor.pin_memory())");
   if (capturing && host)
     fail(rescclInvalidUsage, "host buffers cannot be captured into a CUDA graph (staged copies)");
-  rescclAlgo* algo = ensure_algo(comm, (Coll)coll);
+  const long long S = (long long)count * elt_size(dt) * (coll == (int)Coll::AllReduce ? 1 : comm->nranks);
+  rescclAlgo* algo = select_algo(comm, (Coll)coll, S);
   if (capturing && (!algo->s->opt.devepoch || algo->s->opt.nvls))
     fail(rescclInvalidUsage, "this algorithm cannot be captured into a CUDA graph (devepoch=0 or nvls=1: "
                              "host-side epochs)");
@@ -1201,6 +1223,7 @@ rescclAlgo* load_algo(rescclComm* comm, const std::string& text) {
   rescclAlgo* raw = algo.get();
   comm->algos.push_back(std::move(algo));
   comm->active[(int)s->ir.coll] = raw;
+  comm->ranked[(int)s->ir.coll].push_back(raw);
   return raw;
 }
 
@@ -1209,6 +1232,17 @@ rescclAlgo* ensure_algo(rescclComm* comm, Coll coll) {
   if (a) return a;
   Ir ir = gen_ring(coll, comm->nranks);
   return load_algo(comm, ir.to_text());
+}
+
+// the algorithm a call of `bytes` (per-rank buffer S) runs: the most recently loaded or
+// activated one of its collective whose [minbytes, maxbytes] holds it; else the active one
+rescclAlgo* select_algo(rescclComm* comm, Coll coll, long long bytes) {
+  const auto& v = comm->ranked[(int)coll];
+  for (auto it = v.rbegin(); it != v.rend(); ++it) {
+    const Options& o = (*it)->s->opt;
+    if (bytes >= o.min_bytes && (o.max_bytes < 0 || bytes <= o.max_bytes)) return *it;
+  }
+  return ensure_algo(comm, coll);
 }
 
 Group* make_group(int dev, int n) {
@@ -1888,6 +1922,9 @@ rescclResult_t rescclSetActiveAlgorithm(rescclComm_t comm, rescclAlgo_t algo) {
   API_BEGIN
   if (!comm || !algo || algo->comm != comm) fail(rescclInvalidArgument, "algorithm does not belong to comm");
   comm->active[(int)algo->s->ir.coll] = algo;
+  auto& v = comm->ranked[(int)algo->s->ir.coll];
+  v.erase(std::remove(v.begin(), v.end(), algo), v.end());
+  v.push_back(algo);
   API_END
 }
 

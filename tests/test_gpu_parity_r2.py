@@ -137,3 +137,35 @@ def test_tb_utilization_trace(name, coll, kw):
         assert 0.0 <= u[k] <= 1.0, (k, u[k])
     exp = replay.replay(lower.lower(g, direct=True), xs, "float32", count, chunk_bytes=1 << 18, instances=2, K=2)
     _check(outs, exp)
+
+
+@pytest.mark.timeout(300)
+def test_size_based_algorithm_selection():
+    """minbytes / maxbytes (include/resccl.h): a full-mesh AllReduce (HM with one node of 8,
+    Fig. 16 at nNodes = 1) serves small calls, the ring large ones; every call is bit-exact
+    against the oracle's replay of the algorithm that served it (the two reduce in
+    different association orders, so a wrong pick shows up as a byte difference)."""
+    import torch
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    from gpu_helpers import to_numpy, to_torch
+    n = 8
+    mesh = oir.generate("hm", "allreduce", n, g=8)
+    ring = oir.generate("ring", "allreduce", n)
+    mesh.extra.update(dict(instances="2", chunkbytes=str(1 << 20), direct="1", maxbytes=str(256 << 10)))
+    ring.extra.update(dict(instances="4", chunkbytes=str(1 << 20), direct="1", minbytes=str((256 << 10) + 1)))
+    grp = R.VirtualGroup(n, 0)
+    try:
+        grp.load(ring.to_text())
+        grp.load(mesh.to_text())
+        for count, g, inst in ((1000, mesh, 2), (64 << 10, mesh, 2), ((64 << 10) + 8, ring, 4), (1 << 20, ring, 4)):
+            xs = inp.all_inputs("float32", 30, n, count)
+            s = [to_torch(x, "float32") for x in xs]
+            r = [torch.empty_like(t) for t in s]
+            grp.allreduce(s, r)
+            torch.cuda.synchronize()
+            assert grp.async_error() == 0
+            exp = replay.replay(lower.lower(g, direct=True), xs, "float32", count, chunk_bytes=1 << 20,
+                                instances=inst, K=4)
+            _check([to_numpy(t, "float32") for t in r], exp)
+    finally:
+        grp.destroy()
