@@ -59,6 +59,9 @@ def parse():
     p.add_argument("--inplace-steps", type=int, default=10,
                    help="also time in-place calls (recv = send) -> config.inplace_busbw_gbs")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--tuned-sweep", default="0.0009765625,0.0625,1,4,16,64,256",
+                   help="MiB-per-rank sizes for the size-tuned AllReduce (mesh / mesh-port schedules selected "
+                        "by minbytes / maxbytes); '' = none")
     p.add_argument("--sweep", default="0.0009765625,1,16,64",
                    help="comma-separated MiB-per-rank sizes for the busBW-vs-size points reported beside the "
                         "headline (slices of the bench buffers; small points are L2-resident); '' = none")
@@ -331,6 +334,7 @@ def main():
              for r in my_ranks}
     recvs = {r: torch.empty_like(sends[r]) for r in my_ranks}
     nvls_state = None
+    win = None
     if multi and args.nvls:
         from paper_conf_sigcomm_liuhlgcwz025_b200.torch_api import tensor_at
         pad = 256 // elt
@@ -453,10 +457,14 @@ def main():
             ims = float(t.item())
         inplace_bus = round(S / (ims * 1e-3) / 1e9 * 2 * (n - 1) / n, 2)
 
-    # ---- extra size sweep (busBW vs size)
-    sweep, sweep_us = {}, {}
-    if args.sweep:
-        for mb in [float(x) for x in args.sweep.split(",") if x]:
+    # ---- extra size sweeps (busBW vs size, device clock)
+    def graph_sweep(cms, sizes_mb):
+        """busBW and time per call for slices of the bench buffers: the calls are captured
+        in one CUDA graph (device-side flag epochs) and replayed, so the host's per-call
+        submission cost (8 virtual ranks x ctypes + runtime calls, ~60 us) does not hide
+        small-message latency."""
+        bus, us = {}, {}
+        for mb in sizes_mb:
             cnt = int(mb * (1 << 20)) // elt
             if cnt > count:
                 continue  # sweep points are slices of the bench buffers
@@ -464,19 +472,16 @@ def main():
             r2 = {r: recvs[r][:cnt] for r in my_ranks}
             for _ in range(3):
                 for r in my_ranks:
-                    (comms[0] if multi else comms[r]).allreduce(s2[r], r2[r], stream=sid)
+                    (cms[0] if multi else cms[r]).allreduce(s2[r], r2[r], stream=sid)
             torch.cuda.synchronize(dev)
             barrier()
-            # device clock: the calls are captured in one CUDA graph (device-side flag epochs)
-            # and replayed, so the host's per-call submission cost (8 virtual ranks x ctypes +
-            # runtime calls, ~60 us) does not hide small-message latency
             reps = 10
             cs = torch.cuda.Stream(dev)
             graph = torch.cuda.CUDAGraph()
             with torch.cuda.graph(graph, stream=cs):
                 for _ in range(reps):
                     for r in my_ranks:
-                        (comms[0] if multi else comms[r]).allreduce(s2[r], r2[r], stream=cs.cuda_stream)
+                        (cms[0] if multi else cms[r]).allreduce(s2[r], r2[r], stream=cs.cuda_stream)
             graph.replay()
             torch.cuda.synchronize(dev)
             barrier()
@@ -494,8 +499,45 @@ def main():
                 t_ms = float(t.item())
             del graph
             lab = f"{round(mb * 1024)}KiB" if mb < 1 else f"{mb:g}MiB"
-            sweep[lab] = round(cnt * elt / (t_ms * 1e-3) / 1e9 * 2 * (n - 1) / n, 2)
-            sweep_us[lab] = round(t_ms * 1e3, 2)
+            bus[lab] = round(cnt * elt / (t_ms * 1e-3) / 1e9 * 2 * (n - 1) / n, 2)
+            us[lab] = round(t_ms * 1e3, 2)
+        return bus, us
+
+    sweep, sweep_us = {}, {}
+    if args.sweep:
+        sweep, sweep_us = graph_sweep(comms, [float(x) for x in args.sweep.split(",") if x])
+
+    # ---- the size-tuned AllReduce (a second communicator set loading several schedules
+    # with minbytes / maxbytes ranges, include/resccl.h): the full mesh of Fig. 16 at one
+    # node of 8 (HM, nNodes = 1: 7 pull-reduces + 1 push per chunk instead of the ring's 14
+    # hops) for small messages, the same mesh under the port link model (one duplex CTA
+    # per rank x instances) above 2 MiB.  r02 geometry sweep: profiles/r02_lat_graph_tuned.jsonl
+    tuned, tuned_us, tuned_table = {}, {}, None
+    if args.tuned_sweep and args.algo == "ring":
+        two = 2 << 20
+        tuned_table = [("hm", "g=8", dict(instances=14, chunkbytes=8 << 20, linkmodel="port", minbytes=(32 << 20) + 1)),
+                       ("hm", "g=8", dict(instances=18, chunkbytes=8 << 20, linkmodel="port", minbytes=two + 1,
+                                          maxbytes=32 << 20)),
+                       ("hm", "g=8", dict(instances=2, chunkbytes=32 << 20, maxbytes=two))]
+        if multi:
+            tcomm = R.init_process_group_comm(rank, world, local)
+            tcomms = [tcomm]
+        else:
+            tgrp = R.VirtualGroup(n, 0)
+            tcomms = tgrp.comms
+        for name, gopt, o in tuned_table:
+            t_text = R.rescclGenerateIr(name, "allreduce", n, gopt)
+            h2, rest2 = t_text.split("\n", 1)
+            h2 += f" nwarps=8 fifodepth=2 direct={direct}" + "".join(f" {k}={v}" for k, v in o.items())
+            for c in tcomms:
+                c.load(h2 + "\n" + rest2)
+        if multi and direct and win is not None and not (nvls_state or "").startswith("nvls"):
+            tcomm.register(win)
+        tuned, tuned_us = graph_sweep(tcomms, [float(x) for x in args.tuned_sweep.split(",") if x])
+        if not multi:
+            tgrp.destroy()
+        else:
+            tcomm.destroy()
 
     if rank != 0:
         if multi:
@@ -598,6 +640,10 @@ def main():
         line["sweep_busbw_gbs"] = sweep  # busBW vs size (BASELINE metric); not the headline value
         line["sweep_us"] = sweep_us      # device-clock time per call (CUDA-graph replay)
         line["sweep_timing"] = "CUDA-graph replay of 10 calls (device clock; host submission excluded)"
+    if tuned:
+        line["tuned_busbw_gbs"] = tuned  # size-tuned schedule selection (mesh / mesh-port)
+        line["tuned_us"] = tuned_us
+        line["tuned_schedules"] = [f"{a} {g} " + " ".join(f"{k}={v}" for k, v in o.items()) for a, g, o in tuned_table]
     print(json.dumps(line), flush=True)
     if multi:
         torch.distributed.destroy_process_group()
