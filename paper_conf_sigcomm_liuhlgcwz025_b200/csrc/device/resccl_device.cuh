@@ -1422,7 +1422,8 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       if (stored == issued) idle_on(L, t_idle);
       else idle_off(L, t_idle);
 #if RESCCL_LOOKAHEAD
-      if (L.wa_c < L.wa_n && stored == issued && (spins & 3) == 0) lookahead(L);  // only while data-idle
+      if (stored == issued && (spins & 3) == 0 && L.wa_c < L.wa_n) lookahead(L);  // only while data-idle
+                                                                                 // (register tests first)
 #endif
       if (stored < issued) {
         // idle with a tile outstanding: sleep on the oldest one's barrier (it is the next
