@@ -51,6 +51,9 @@ def parse():
     p.add_argument("--nwarps", type=int, default=0)
     p.add_argument("--tma", type=int, default=-1, help="-1 = library default (on)")
     p.add_argument("--direct", type=int, default=-1, help="direct push/pull transport (default 1; N>1 registers a symmetric window)")
+    p.add_argument("--pushreduce", type=int, default=0,
+                   help="with the direct transport: push rrc operands into the receiver's FIFO instead of pulling "
+                        "them (DESIGN R31)")
     p.add_argument("--nvls", type=int, default=0,
                    help="f3: N>1 only -- send/recv in an NVLS window, NVLS kernel (falls back to --direct if "
                         "the fabric refuses multicast)")
@@ -311,7 +314,8 @@ def main():
             "nwarps": args.nwarps or ((8 if not multi else 16) if tuned else None),
             "tma": None if args.tma < 0 else args.tma,
             "tmastages": 2 if tuned else None, "tmatile": 24576 if tuned else None,
-            "direct": direct, "nvls": 1 if (args.nvls and multi) else None}
+            "direct": direct, "nvls": 1 if (args.nvls and multi) else None,
+            "pushreduce": 1 if (args.pushreduce and direct) else None}
     text = ir_text(R, args.algo, n, opts)
 
     if multi:

@@ -146,11 +146,15 @@ def _greedy_merge(conns_act: Dict[Tuple[int, str], set]) -> List[List[Tuple[int,
     return groups
 
 
-def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool = False) -> Plan:
+def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool = False,
+          pushreduce: bool = False) -> Plan:
     """``direct`` (reading R23): no FIFO staging; recv tasks are pushed into the
     receiver's location after it posts "writable", rrc tasks are pulled from the
     sender's location, whose completion is the receiver's read acknowledgement.
-    Fusion in direct mode chains a receive with the next hop's push or "readable"."""
+    Fusion in direct mode chains a receive with the next hop's push or "readable".
+    ``pushreduce`` (with ``direct``, DESIGN R31): rrc tasks keep the staged FIFO (the
+    sender pushes its operand into the receiver's slot, the receiver reduces locally);
+    recv tasks stay direct pushes.  Only primitives of the same mode fuse."""
     edges, edge_rank = build_dag(ir)
     check_defined_reads(ir)
     if Pr is None:
@@ -189,7 +193,9 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
                   store=True, dst_buf=write_buf(coll, t.dst, t.chunk),
                   src_buf=read_buf(t.dst, t.chunk, t.step) if t.op == RRC else None)
         if direct:
-            if t.op == RRC:
+            if t.op == RRC and pushreduce:
+                pass                                   # staged push-reduce (R31)
+            elif t.op == RRC:
                 s.direct = s.pull = rv.direct = rv.pull = True
                 s.kind, rv.kind = "psend", "prrc"
                 rv.rem_buf = s.src_buf
@@ -241,7 +247,7 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
             recv_lane = sorted((p for p in ps if p.lane == "R"), key=lambda p: (p.cta, p.pc))
             taken = set()
             for a in recv_lane:
-                cands = [b for b in ps if b.lane == "S" and b.cta == a.cta
+                cands = [b for b in ps if b.lane == "S" and b.cta == a.cta and b.direct == a.direct
                          and b.pid not in taken and deps[r][b.pid] == {a.pid}]
                 if not cands:
                     continue
@@ -279,7 +285,7 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
                         break
                 store = (final and is_output(coll, r, a.chunk)) or readers != {t2}
                 a.send_task = t2
-                if direct:       # value stays in our location; the send part keeps its mode
+                if a.direct:     # value stays in our location; the send part keeps its mode
                     a.kind = DIRECT_FUSED[(a.kind, b.kind)]
                     a.rem_out = b.rem_out
                     if a.kind.startswith("drecv"):
@@ -365,6 +371,7 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
     plan = Plan(ir, model, edges, edge_rank, Pr, pidx, out_prims, lanes,
                 send_groups, recv_groups,
                 {r: len(act[r]) for r in range(N)}, any_fused, direct)
+    plan.pushreduce = bool(direct and pushreduce)
     plan._act = act
     if fuse and any(absorbed[r] for r in range(N)):
         from .replay import deadlock_free
@@ -373,6 +380,7 @@ def lower(ir: IR, model: str = "pair", fuse: bool = True, Pr=None, direct: bool 
             op, ln = build(ab)
             pl = Plan(ir, model, edges, edge_rank, Pr, pidx, op, ln, send_groups, recv_groups,
                       {r: len(act[r]) for r in range(N)}, fused, direct)
+            pl.pushreduce = bool(direct and pushreduce)
             pl._act = act
             return pl
 

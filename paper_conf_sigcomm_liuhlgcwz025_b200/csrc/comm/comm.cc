@@ -146,6 +146,7 @@ struct Options {
   int lookahead = 1;     // DESIGN R30: "writable" credits posted ahead of the lane (1: TMA variant, 2: both)
   int sched = 0;     // 0 = HPDS (Alg. 1), 1 = round-robin baseline
   int direct = 0;    // direct transport (R23): virtual ranks / single-process only
+  int pushreduce = 0;  // with direct: rrc tasks keep the staged FIFO -- push-reduce (R31)
   int l2hint = 1;
   int tma_min = 32768;   // r01 (24 KiB tiles): the TMA engine wins from 32 KiB slices (16 MiB AR +31%)
   int backoff = 1;
@@ -211,6 +212,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "prefetch") o.prefetch = (int)to_long(v, k);
   else if (k == "tmamin") o.tma_min = (int)to_long(v, k);
   else if (k == "direct") o.direct = (int)to_long(v, k);
+  else if (k == "pushreduce") o.pushreduce = (int)to_long(v, k);
   else if (k == "backoff") o.backoff = (int)to_long(v, k);
   else if (k == "pollacq") o.pollacq = (int)to_long(v, k);
   else if (k == "jitter") o.jitter = (int)to_long(v, k);
@@ -270,9 +272,9 @@ Plan lower_with(const Ir& ir, LinkModel m, const Options& o) {
   if (o.sched == 1) {
     Dag d = build_dag(ir);
     auto pr = round_robin(ir, d, m);
-    return lower(ir, m, o.fuse, &pr, o.direct != 0);
+    return lower(ir, m, o.fuse, &pr, o.direct != 0, o.pushreduce != 0);
   }
-  return lower(ir, m, o.fuse, nullptr, o.direct != 0);
+  return lower(ir, m, o.fuse, nullptr, o.direct != 0, o.pushreduce != 0);
 }
 
 Plan make_plan(const Ir& ir, Options& o) {
@@ -529,7 +531,7 @@ std::string info_json(const AlgoShared& a) {
   o << "{\"plan\":" << pj << ",\"instances\":" << a.opt.instances << ",\"chunkbytes\":" << a.opt.chunk_bytes
     << ",\"fifodepth\":" << a.opt.fifo_depth << ",\"nwarps\":" << a.opt.nwarps << ",\"tma\":" << a.opt.tma
     << ",\"tmatile\":" << a.opt.tma_tile << ",\"tmastages\":" << a.opt.tma_stages << ",\"l2hint\":" << a.opt.l2hint << ",\"prefetch\":" << a.opt.prefetch << ",\"sched\":\""
-    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"bulkred\":" << a.opt.bulkred << ",\"devepoch\":" << a.opt.devepoch << ",\"nvls\":" << a.opt.nvls << ",\"nvlsctas\":" << a.opt.nvls_ctas << ",\"linkmodel\":\""
+    << (a.opt.sched ? "rr" : "hpds") << "\",\"direct\":" << a.opt.direct << ",\"pushreduce\":" << a.opt.pushreduce << ",\"bulkred\":" << a.opt.bulkred << ",\"devepoch\":" << a.opt.devepoch << ",\"nvls\":" << a.opt.nvls << ",\"nvlsctas\":" << a.opt.nvls_ctas << ",\"linkmodel\":\""
     << (a.opt.model == LinkModel::Pair ? "pair" : "port") << "\",\"region_bytes\":" << a.lay.region_bytes
     << ",\"ctas\":[";
   for (size_t r = 0; r < a.lay.ctas.size(); ++r) o << (r ? "," : "") << a.lay.ctas[r];
@@ -2207,7 +2209,7 @@ rescclResult_t rescclProfilePlanner(const char* program, const char* opts, int v
   auto t2 = clk::now();
   auto pr = o.sched ? round_robin(ir, d, o.model) : hpds(ir, d, o.model);  // Scheduling
   auto t3 = clk::now();
-  Plan p = lower(ir, o.model, false, &pr, o.direct != 0);  // Lowering (translation + TB allocation)
+  Plan p = lower(ir, o.model, false, &pr, o.direct != 0, o.pushreduce != 0);  // Lowering (translation + TB allocation)
   Layout L = make_layout(p, o.fifo_depth, o.instances, o.chunk_bytes);
   CodegenOpts co = codegen_opts(o);
   co.rank_lo = 0;

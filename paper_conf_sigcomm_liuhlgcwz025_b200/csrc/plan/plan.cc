@@ -296,7 +296,7 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
       bool store = (final_ && is_output(ir.coll, r, a.chunk)) || readers != std::set<int>{t2};
       a.send_task = t2;
       a.flags |= kSend;
-      if (P.direct) {
+      if (a.flags & kDirect) {
         // direct: the next hop pulls from / is pushed from our location, so the value
         // stays stored; the send part keeps its push / pull mode
         a.flags |= (b.flags & kSendPull);
@@ -404,11 +404,13 @@ static void build_ranks(Plan& P, const std::vector<Raw>& raw, const std::vector<
   }
 }
 
-Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<int>>* pr_in, bool direct) {
+Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<int>>* pr_in, bool direct,
+           bool pushreduce) {
   Plan P;
   P.ir = ir;
   P.model = m;
   P.direct = direct;
+  P.pushreduce = direct && pushreduce;
   P.dag = build_dag(ir);
   P.pr = pr_in ? *pr_in : hpds(ir, P.dag, m);
   const int T = (int)ir.t.size(), N = ir.nranks;
@@ -471,7 +473,7 @@ Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<i
     rv.dst_buf = write_buf(ir.coll, x.dst, x.chunk);
     rv.src_buf = x.op == Op::Rrc ? read_buf(x.dst, x.chunk, x.step) : BufNone;
     rv.lane = 1;
-    if (direct) {
+    if (direct && !(x.op == Op::Rrc && pushreduce)) {  // (push-reduce, R31: rrc tasks stay staged)
       if (x.op == Op::Rrc) {  // pull: receiver reads the sender's location
         s.flags |= kDirect | kSendPull;
         rv.flags |= kDirect | kPull;
@@ -535,6 +537,7 @@ Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<i
         int best = -1;
         for (int b = 0; b < (int)ps.size(); ++b) {
           if (ps[b].lane != 0 || ps[b].cta != ps[a].cta || taken.count(b)) continue;
+          if ((ps[b].flags & kDirect) != (ps[a].flags & kDirect)) continue;  // only same-mode pairs fuse
           if (raw[r].deps[b] != std::set<int>{a}) continue;
           if (best < 0 || std::make_pair(ps[b].pc, ir.t[ps[b].send_task].dst) <
                               std::make_pair(ps[best].pc, ir.t[ps[best].send_task].dst))
@@ -717,7 +720,8 @@ std::string plan_json(const Plan& P) {
   const Ir& ir = P.ir;
   o << "{\"name\":\"" << ir.name << "\",\"coll\":\"" << coll_name(ir.coll) << "\",\"nranks\":" << ir.nranks
     << ",\"model\":\"" << (P.model == LinkModel::Pair ? "pair" : "port") << "\",\"fused\":"
-    << (P.fused ? "true" : "false") << ",\"direct\":" << (P.direct ? "true" : "false") << ",\"n_edges\":" << P.dag.edges.size() << ",\"tasks\":[";
+    << (P.fused ? "true" : "false") << ",\"direct\":" << (P.direct ? "true" : "false")
+    << ",\"pushreduce\":" << (P.pushreduce ? "true" : "false") << ",\"n_edges\":" << P.dag.edges.size() << ",\"tasks\":[";
   for (size_t i = 0; i < ir.t.size(); ++i) {
     auto& x = ir.t[i];
     o << (i ? "," : "") << "[" << x.src << "," << x.dst << "," << x.step << "," << x.chunk << ",\""

@@ -99,13 +99,14 @@ struct Plan {
   std::vector<RankPlan> ranks;
   bool fused = false;
   bool direct = false;
+  bool pushreduce = false;  // direct plan whose rrc tasks keep the staged FIFO (R31)
   // FIFO order of every link: tasks sorted by pipeline index
   std::vector<int> link_pos;  // task -> position on its link
   std::vector<int> link_len;  // task -> #tasks on its link
 };
 
 Plan lower(const Ir& ir, LinkModel m, bool fuse, const std::vector<std::vector<int>>* pr = nullptr,
-           bool direct = false);
+           bool direct = false, bool pushreduce = false);
 
 // Control-only blocking simulation of the lowered plan (I4).  Returns true if every
 // lane completes for FIFO depth K and n_mb micro-batches.

@@ -195,6 +195,10 @@ def _window_worker(rank, world, port, algo, coll, count, dtype, q, opts):
     ("ring", "reducescatter", 2, 9000, "chunkbytes=4096 instances=2 fifodepth=2 direct=1"),
     ("dbt", "allreduce", 4, 9000, "chunkbytes=4096 instances=2 fifodepth=2 direct=1"),
     ("ring", "allreduce", 2, (6 << 20) + 33, "chunkbytes=4194304 instances=2 fifodepth=2 direct=1"),
+    # push-reduce (R31): rrc operands pushed into the receiver's FIFO, recv payloads pushed directly
+    ("ring", "allreduce", 2, 9000, "chunkbytes=4096 instances=2 fifodepth=2 direct=1 pushreduce=1"),
+    ("dbt", "allreduce", 4, 9000, "chunkbytes=4096 instances=2 fifodepth=2 direct=1 pushreduce=1"),
+    ("ring", "allreduce", 2, (6 << 20) + 33, "chunkbytes=4194304 instances=2 fifodepth=2 direct=1 pushreduce=1"),
 ])
 def test_ipc_registered_windows_direct(algo, coll, world, count, opts):
     import torch.multiprocessing as mp

@@ -169,3 +169,26 @@ def test_size_based_algorithm_selection():
             _check([to_numpy(t, "float32") for t in r], exp)
     finally:
         grp.destroy()
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("name,coll,kw", [("ring", "allreduce", {}), ("hm", "allreduce", {"g": 4}),
+                                          ("dbt", "allreduce", {}), ("synth", "reducescatter", {"seed": 1, "fanout": 3}),
+                                          ("ring", "allgather", {}), ("hm", "allreduce", {"g": 8})])
+@pytest.mark.parametrize("count,cb", [(3 * 4096 + 77, 4096), ((2 << 20) + 4099, 1 << 20)])
+def test_pushreduce_bit_exact(name, coll, kw, count, cb):
+    """Push-reduce variant of the direct transport (R31): the sender pushes
+    rrc operands into the receiver's FIFO slot (staged) while recv payloads are pushed
+    straight into the receiver's location; register path and TMA engine."""
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    n = 8
+    g = oir.generate(name, coll, n, **kw)
+    for k, v in dict(chunkbytes=cb, instances=2, fifodepth=2, direct=1, pushreduce=1).items():
+        g.extra[k] = str(v)
+    m = count * n if coll == "reducescatter" else count
+    xs = inp.all_inputs("float32", 25, n, m)
+    outs, info, err = run_virtual(R, g.to_text(), coll, xs, "float32", count)
+    assert err == 0 and info["pushreduce"] == 1
+    exp = replay.replay(lower.lower(g, direct=True, pushreduce=True), xs, "float32", count, chunk_bytes=cb,
+                        instances=2, K=2)
+    _check(outs, exp)

@@ -147,3 +147,24 @@ def test_round_robin_differs_from_hpds_on_dbt8():
     edges, _ = dag.build_dag(g)
     assert [len(p) for p in hpds.round_robin(g, edges)] == [24, 16, 16, 16, 4, 12, 12, 12]
     assert [len(p) for p in hpds.hpds(g, edges)] == [24, 24, 24, 24, 4, 4, 4, 4]
+
+
+@pytest.mark.parametrize("name,coll,n,kw", ALGOS)
+def test_pushreduce_replay_definition_races_deadlock(name, coll, n, kw):
+    """R31 plans: int32 results equal the definition, the happens-before check finds no
+    race (a staged slot and a direct push share one link's credit counter and flag ring),
+    and the blocking model completes."""
+    from oracle import definition
+    g = oir.generate(name, coll, n, **kw)
+    pl = lower.lower(g, direct=True, pushreduce=True)
+    count = 3000 + 7
+    xs = inp.all_inputs("int32", 5, n, count * (n if coll == "reducescatter" else 1), mode="wrap")
+    for inplace in (False, True):
+        got = replay.replay(pl, xs, "int32", count, chunk_bytes=2048, instances=2, K=2, inplace=inplace)
+        ref = {"allreduce": definition.allreduce, "allgather": lambda x, d: definition.allgather(x),
+               "reducescatter": definition.reducescatter}[coll](xs, "int32")
+        for r in range(n):
+            assert np.array_equal(got[r], ref[r]), (inplace, r)
+    for K, nmb in ((1, 2), (2, 3)):
+        assert replay.happens_before_races(pl, n_mb=nmb, instances=1, K=K) == []
+    assert replay.deadlock_free(pl, Ks=(1, 2), n_mbs=(1, 2, 3, 16))

@@ -237,3 +237,21 @@ def test_direct_plan_matches_oracle(name, coll, n, kw, model):
     for K, nmb in ((1, 1), (1, 3), (2, 16)):
         assert R.rescclCheckDeadlock(g.to_text(), f"linkmodel={model} direct=1", K, nmb) == \
             replay.deadlock_free(pl, Ks=(K,), n_mbs=(nmb,))
+
+
+@pytest.mark.parametrize("name,coll,n,kw", CASES)
+@pytest.mark.parametrize("model", ["pair", "port"])
+def test_pushreduce_plan_matches_oracle(name, coll, n, kw, model):
+    """Push-reduce variant of the direct transport (R31): rrc tasks keep the staged FIFO,
+    recv tasks stay direct pushes; same lowering in the C++ planner and the oracle, and the
+    same deadlock verdicts."""
+    g = _oracle_ir(name, coll, n, kw)
+    js = R.rescclPlanIr(g.to_text(), f"linkmodel={model} direct=1 pushreduce=1")
+    pl = lower.lower(g, model, direct=True, pushreduce=True)
+    assert js["plan"]["pushreduce"] is True and pl.pushreduce
+    assert _norm_cpp(js) == _norm_oracle(pl)
+    kinds = {p["kind"] for rp in js["plan"]["ranks"] for p in rp["prims"]}
+    assert not kinds & {"psend", "prrc", "prrc_p", "prrc_d"}   # nothing is pulled
+    for K, nmb in ((1, 1), (1, 3), (2, 16)):
+        assert R.rescclCheckDeadlock(g.to_text(), f"linkmodel={model} direct=1 pushreduce=1", K, nmb) == \
+            replay.deadlock_free(pl, Ks=(K,), n_mbs=(nmb,))
