@@ -51,6 +51,9 @@ def parse():
     p.add_argument("--nwarps", type=int, default=0)
     p.add_argument("--tma", type=int, default=-1, help="-1 = library default (on)")
     p.add_argument("--direct", type=int, default=-1, help="direct push/pull transport (default 1; N>1 registers a symmetric window)")
+    p.add_argument("--nccl-compare", type=int, default=1,
+                   help="N>1: also report a traced call's TB utilisation and NCCL's same-size AllReduce (busBW, "
+                        "channels)")
     p.add_argument("--pushreduce", type=int, default=0,
                    help="with the direct transport: push rrc operands into the receiver's FIFO instead of pulling "
                         "them (DESIGN R31)")
@@ -519,10 +522,13 @@ def main():
     tuned, tuned_us, tuned_table = {}, {}, None
     if args.tuned_sweep and args.algo == "ring":
         two = 2 << 20
-        tuned_table = [("hm", "g=8", dict(instances=14, chunkbytes=8 << 20, linkmodel="port", minbytes=(32 << 20) + 1)),
-                       ("hm", "g=8", dict(instances=18, chunkbytes=8 << 20, linkmodel="port", minbytes=two + 1,
-                                          maxbytes=32 << 20)),
-                       ("hm", "g=8", dict(instances=2, chunkbytes=32 << 20, maxbytes=two))]
+        mesh = f"g={n}"  # the hierarchical mesh at one node of all n ranks: a full mesh
+        i_big, i_mid = (14, 18) if not multi else (24, 24)
+        tuned_table = [("hm", mesh, dict(instances=i_big, chunkbytes=8 << 20, linkmodel="port",
+                                         minbytes=(32 << 20) + 1)),
+                       ("hm", mesh, dict(instances=i_mid, chunkbytes=8 << 20, linkmodel="port", minbytes=two + 1,
+                                         maxbytes=32 << 20)),
+                       ("hm", mesh, dict(instances=2, chunkbytes=32 << 20, maxbytes=two))]
         if multi:
             tcomm = R.init_process_group_comm(rank, world, local)
             tcomms = [tcomm]
@@ -542,6 +548,62 @@ def main():
             tgrp.destroy()
         else:
             tcomm.destroy()
+
+    # ---- N > 1 evidence: TB utilisation of one traced call of the same
+    # algorithm, and NCCL's AllReduce of the same buffer on the same GPUs -- its busBW and
+    # its channel count (NCCL_DEBUG=INFO, one CTA per channel) as the "SMs vs NCCL"
+    # denominator.  Every rank runs both (collectives); failures are recorded, not fatal.
+    multi_extra = {}
+    if multi and args.nccl_compare:
+        try:
+            tt = R.rescclGenerateIr(args.algo, "allreduce", n, "g=4" if args.algo == "hm" else "")
+            h3, rest3 = tt.split("\n", 1)
+            h3 += "".join(f" {k}={v}" for k, v in opts.items() if v is not None) + " trace=1"
+            ta = comm.load(h3 + "\n" + rest3)
+            comm.allreduce(sends[rank], recvs[rank], stream=sid)
+            torch.cuda.synchronize(dev)
+            u = R.rescclGetTbUtilization(ta)
+            multi_extra["tb_utilization"] = {k: round(u[k], 4) if isinstance(u[k], float) else u[k]
+                                             for k in ("tbs", "comm_time", "avg_idle", "max_idle", "ctas",
+                                                       "cta_comm_time", "cta_avg_idle", "cta_max_idle")}
+        except Exception as e:  # noqa: BLE001
+            multi_extra["tb_utilization"] = {"error": str(e)[:300]}
+        nccl_log = f"/tmp/resccl_bench_nccl.{os.getpid()}.log"
+        try:
+            import re as _re
+            os.environ["NCCL_DEBUG"] = "INFO"
+            os.environ["NCCL_DEBUG_SUBSYS"] = "INIT,TUNING"
+            os.environ["NCCL_DEBUG_FILE"] = nccl_log
+            ng = torch.distributed.new_group(backend="nccl")
+            xb = sends[rank].clone()
+            for _ in range(3):
+                torch.distributed.all_reduce(xb, group=ng)
+            torch.cuda.synchronize(dev)
+            barrier()
+            n0 = torch.cuda.Event(enable_timing=True)
+            n1 = torch.cuda.Event(enable_timing=True)
+            n0.record()
+            for _ in range(10):
+                torch.distributed.all_reduce(xb, group=ng)
+            n1.record()
+            torch.cuda.synchronize(dev)
+            nms = n0.elapsed_time(n1) / 10
+            t = torch.tensor([nms], dtype=torch.float64)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            nms = float(t.item())
+            chan = None
+            try:
+                txt = open(nccl_log).read()
+                m = _re.findall(r"(\d+) coll channels", txt) or _re.findall(r"Channel \d+/(\d+)", txt)
+                chan = int(m[-1]) if m else None
+            except OSError:
+                pass
+            multi_extra["nccl"] = {"busbw_gbs": round(S / (nms * 1e-3) / 1e9 * 2 * (n - 1) / n, 2),
+                                   "ms": round(nms, 4), "channels": chan,
+                                   "ctas_note": "NCCL runs one CTA per channel",
+                                   "resccl_ctas_per_rank": blocks[rank]}
+        except Exception as e:  # noqa: BLE001
+            multi_extra["nccl"] = {"error": str(e)[:300]}
 
     if rank != 0:
         if multi:
@@ -644,6 +706,8 @@ def main():
         line["sweep_busbw_gbs"] = sweep  # busBW vs size (BASELINE metric); not the headline value
         line["sweep_us"] = sweep_us      # device-clock time per call (CUDA-graph replay)
         line["sweep_timing"] = "CUDA-graph replay of 10 calls (device clock; host submission excluded)"
+    if multi_extra:
+        line["multi_gpu"] = multi_extra
     if tuned:
         line["tuned_busbw_gbs"] = tuned  # size-tuned schedule selection (mesh / mesh-port)
         line["tuned_us"] = tuned_us
