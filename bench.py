@@ -528,7 +528,7 @@ def main():
                                          minbytes=(32 << 20) + 1)),
                        ("hm", mesh, dict(instances=i_mid, chunkbytes=8 << 20, linkmodel="port", minbytes=two + 1,
                                          maxbytes=32 << 20)),
-                       ("hm", mesh, dict(instances=2, chunkbytes=32 << 20, maxbytes=two))]
+                       ("hm", mesh, dict(instances=2, chunkbytes=two, maxbytes=two))]
         if multi:
             tcomm = R.init_process_group_comm(rank, world, local)
             tcomms = [tcomm]
