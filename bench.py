@@ -316,7 +316,11 @@ def main():
             "fifodepth": args.fifo_depth or 2,
             "nwarps": args.nwarps or ((8 if not multi else 16) if tuned else None),
             "tma": None if args.tma < 0 else args.tma,
-            "tmastages": 2 if tuned else None, "tmatile": 24576 if tuned else None,
+            "tmastages": 2 if tuned else None,
+            # 28 KiB tiles with 16 warps: 94 GB/s of HBM per SM at 8 CTAs against 85 with 24 KiB
+            # (profiles/r02_per_sm_rate.jsonl) -- what counts at N>1, where few CTAs per rank
+            # must carry NVLink; the HBM-bound N=1 headline is equal either way (320 GB/s)
+            "tmatile": (24576 if not multi else 28672) if tuned else None,
             "direct": direct, "nvls": 1 if (args.nvls and multi) else None,
             "pushreduce": 1 if (args.pushreduce and direct) else None}
     text = ir_text(R, args.algo, n, opts)

@@ -256,8 +256,8 @@ Options make_options(const Ir& ir, const char* extra) {
   if (o.chunk_bytes < 256 || o.chunk_bytes > (1ll << 30)) fail(rescclInvalidArgument, "chunkbytes out of range");
   if (o.nwarps < 2 || o.nwarps > 32 || o.nwarps % 2) fail(rescclInvalidArgument, "nwarps must be even, 2..32");
   if (o.tma_tile < 1024 || o.tma_tile % 128 || o.tma_stages < 1 || o.tma_stages > 8 ||
-      4 * o.tma_tile * o.tma_stages > 200 * 1024)
-    fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 4*tile*stages <= 200 KiB");
+      4 * o.tma_tile * o.tma_stages > 224 * 1024)
+    fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 4*tile*stages <= 224 KiB");
   if (o.nvls_ctas < 1 || o.nvls_ctas > 148) fail(rescclInvalidArgument, "nvlsctas must be 1..148");
   if (o.bulkred < 0) o.bulkred = ir.coll == Coll::AllReduce ? 1 : 0;
   if (o.store_lag < 1 || o.store_lag > o.tma_stages)
