@@ -163,6 +163,9 @@ rescclResult_t rescclCommGetAsyncError(rescclComm_t comm, rescclResult_t* err);
  *     algo name=<s> coll=<allgather|reducescatter|allreduce> nranks=<N> nchunks=<N>
  *          [nwarps=16] [instances=1] [chunkbytes=1048576] [fifodepth=4]
  *          [linkmodel=pair|port] [fuse=1] [tbbudget=B]
+ *     tbbudget=B (TBs = CTAs per rank): instances = floor(B / T_min) under the
+ *     pair link model, or the port model (one duplex CTA per rank) with B instances when
+ *     B < T_min or when linkmodel=port is given explicitly.
  *     t <src> <dst> <step> <chunk> <recv|rrc>
  * Environment overrides: RESCCL_INSTANCES, RESCCL_CHUNK_BYTES, RESCCL_FIFO_DEPTH,
  * RESCCL_NWARPS, RESCCL_LINK_MODEL, RESCCL_FUSE, RESCCL_TB_BUDGET.

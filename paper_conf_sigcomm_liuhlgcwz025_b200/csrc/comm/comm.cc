@@ -134,6 +134,7 @@ struct Options {
   int fifo_depth = 4;
   int nwarps = 16;                // Table 2
   LinkModel model = LinkModel::Pair;
+  bool model_set = false;  // linkmodel given explicitly (a TB budget then keeps it)
   bool fuse = true;
   int tb_budget = 0;
   int tma = 1;
@@ -236,6 +237,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
     if (v == "pair") o.model = LinkModel::Pair;
     else if (v == "port") o.model = LinkModel::Port;
     else fail(rescclInvalidArgument, "linkmodel must be pair|port");
+    o.model_set = true;
   }
 }
 
@@ -278,6 +280,14 @@ Plan lower_with(const Ir& ir, LinkModel m, const Options& o) {
 }
 
 Plan make_plan(const Ir& ir, Options& o) {
+  if (o.tb_budget > 0 && o.model_set && o.model == LinkModel::Port) {
+    // explicit port model under a TB budget: one duplex CTA per rank x B instances
+    Plan q = lower_with(ir, LinkModel::Port, o);
+    int t1 = 1;
+    for (auto& r : q.ranks) t1 = std::max(t1, (int)r.ctas.size());
+    o.instances = std::max(1, o.tb_budget / t1);
+    return q;
+  }
   if (o.tb_budget > 0) {
     Plan p = lower_with(ir, LinkModel::Pair, o);
     int tmin = 1;

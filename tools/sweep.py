@@ -94,11 +94,14 @@ if "c3" in which:
     # TB budget B = CTAs per rank (instances = floor(B / T_min) under the pair model, the
     # port model below T_min); each schedule's best transfer chunk of the r02 geometry
     # sweep (DBT 8 MiB, HM 1 MiB), 256-thread CTAs
-    for name, g, cb in (("dbt", "", 8 << 20), ("hm", "g=4", 1 << 20)):
+    for name, g, cb, lm in (("dbt", "", 8 << 20, None), ("hm", "g=4", 1 << 20, None), ("dbt", "", 8 << 20, "port"),
+                            ("hm", "g=4", 1 << 20, "port")):
         for budget in (1, 2, 4, 8, 12, 16, 18):
             for S in (64 << 20, 256 << 20):
-                emit(measure(name, "allreduce", g, dict(chunkbytes=cb, fifodepth=2, tbbudget=budget, nwarps=8,
-                                                        direct=BASE["direct"]), S))
+                o = dict(chunkbytes=cb, fifodepth=2, tbbudget=budget, nwarps=8, direct=BASE["direct"])
+                if lm:
+                    o["linkmodel"] = lm
+                emit(measure(name, "allreduce", g, o, S))
     for S in (64 << 20, 256 << 20):
         emit(measure("ring", "allreduce", "", dict(chunkbytes=1 << 20, fifodepth=2, instances=2,
                                                    direct=BASE["direct"]), S))
