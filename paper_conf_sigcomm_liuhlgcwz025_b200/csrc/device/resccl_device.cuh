@@ -87,21 +87,39 @@ __device__ __forceinline__ void cta_sync() { asm volatile("barrier.sync 0;" ::: 
 // the next launch of the plan.
 __device__ __forceinline__ const KArgs* epochs_begin(const KArgs& a, KArgs* sh) {
   if (!a.epochs) return &a;
+  // thread 0 issues the two epoch loads first (their latency overlaps the copy); every
+  // thread copies a slice of the kernel arguments into shared memory
+  u64 v0 = 0, v1 = 0;
   if (threadIdx.x == 0) {
-    *sh = a;
-    u64 mb, ep;
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(mb) : "l"(&a.epochs[0]) : "memory");
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(ep) : "l"(&a.epochs[1]) : "memory");
-    sh->mb_base = mb;
-    sh->epoch = ep;
-    const unsigned long long old = atomicAdd((unsigned long long*)&a.epochs[2], 1ull);
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v0) : "l"(&a.epochs[0]) : "memory");
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v1) : "l"(&a.epochs[1]) : "memory");
+  }
+  {
+    const u64* src = (const u64*)&a;
+    u64* dst = (u64*)sh;
+    for (int i = threadIdx.x; i < (int)(sizeof(KArgs) / 8); i += blockDim.x) dst[i] = src[i];
+  }
+  cta_sync();
+  if (threadIdx.x == 0) {
+    sh->mb_base = v0;
+    sh->epoch = v1;
+  }
+  cta_sync();
+  // one thread of warp 1 counts this CTA in (its operand depends on the epoch values, so
+  // the arrival cannot be performed before thread 0's loads returned -- they reached
+  // shared memory before the barrier); the last CTA to arrive advances the epochs.  Warp
+  // 0's leader starts its lane without waiting for the round trip.
+  if (threadIdx.x == 32 || (blockDim.x <= 32 && threadIdx.x == 0)) {
+    const u64 mb = sh->mb_base, ep = sh->epoch;
+    u64 z;
+    asm volatile("xor.b64 %0, %1, %1;" : "=l"(z) : "l"(mb ^ ep));
+    const unsigned long long old = atomicAdd((unsigned long long*)&a.epochs[2], 1ull + z);
     if (old == (unsigned long long)gridDim.x - 1) {
       a.epochs[0] = mb + (u64)a.n_mb;
       a.epochs[1] = ep + 1;
       a.epochs[2] = 0;
     }
   }
-  cta_sync();
   return sh;
 }
 __device__ __forceinline__ void epochs_end(const KArgs&) {}

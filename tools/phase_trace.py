@@ -24,6 +24,7 @@ import paper_conf_sigcomm_liuhlgcwz025_b200 as R  # noqa: E402
 
 N = int(os.environ.get("PHASE_N", "8"))
 ALGO = os.environ.get("PHASE_ALGO", "ring")
+GOPTS = os.environ.get("PHASE_GOPTS", "g=4" if ALGO == "hm" else "")
 OPTS = os.environ.get("PHASE_OPTS", "instances=14 nwarps=8 chunkbytes=33554432 fifodepth=2 direct=1")
 
 
@@ -140,7 +141,7 @@ def per_kind(lanes, plan):
 
 def main():
     sizes = [int(x) for x in sys.argv[1:]] or [1024, 1 << 20, 16 << 20]
-    text = R.rescclGenerateIr(ALGO, "allreduce", N, "g=4" if ALGO == "hm" else "")
+    text = R.rescclGenerateIr(ALGO, "allreduce", N, GOPTS)
     hdr, rest = text.split("\n", 1)
     for S in sizes:
         grp = R.VirtualGroup(N, 0)
