@@ -8,6 +8,10 @@ import paper_conf_sigcomm_liuhlgcwz025_b200 as R
 
 N = 8
 M = int(sys.argv[1]) if len(sys.argv) > 1 else 8192
+ALGO = os.environ.get("OVERLAP_ALGO", "ring")
+GOPTS = os.environ.get("OVERLAP_GOPTS", "")
+OPTS = os.environ.get("OVERLAP_OPTS", "chunkbytes=4194304 direct=1")
+INSTS = [int(x) for x in os.environ.get("OVERLAP_INSTANCES", "1,2,4,8,18").split(",")]
 a = torch.randn(M, M, device="cuda:0", dtype=torch.bfloat16)
 b = torch.randn(M, M, device="cuda:0", dtype=torch.bfloat16)
 c = torch.empty(M, M, device="cuda:0", dtype=torch.bfloat16)
@@ -35,11 +39,12 @@ alone = flops * 40 / (e0.elapsed_time(e1) * 1e-3) / 1e12
 print(json.dumps({"gemm_alone_tflops": round(alone, 1), "M": M}), flush=True)
 
 cnt = 25 * (1 << 20) // 2
-for inst in (1, 2, 4, 8, 18):
-    text = R.rescclGenerateIr("ring", "allreduce", N)
+for inst in INSTS:
+    text = R.rescclGenerateIr(ALGO, "allreduce", N, GOPTS)
     h, rest = text.split("\n", 1)
     grp = R.VirtualGroup(N, 0)
-    grp.load(h + f" instances={inst} chunkbytes=4194304 direct=1\n" + rest)
+    grp.load(h + f" instances={inst} {OPTS}\n" + rest)
+    info = grp.plan_info()
     s = [torch.randn(cnt, device="cuda:0").to(torch.bfloat16) for _ in range(N)]
     r = [torch.empty_like(x) for x in s]
     for _ in range(3):
@@ -62,7 +67,8 @@ for inst in (1, 2, 4, 8, 18):
     torch.cuda.synchronize()
     conc = flops * 40 / (g0.elapsed_time(g1) * 1e-3) / 1e12
     ar_conc = f0.elapsed_time(f1) / 40
-    print(json.dumps({"instances": inst, "comm_ctas": N * inst, "gemm_concurrent_tflops": round(conc, 1),
+    print(json.dumps({"algo": ALGO, "gopts": GOPTS, "opts": OPTS, "instances": inst,
+                      "comm_ctas": sum(info["blocks_per_rank"]), "gemm_concurrent_tflops": round(conc, 1),
                       "gemm_slowdown_pct": round(100 * (1 - conc / alone), 2), "ar_alone_us": round(ar_alone * 1e3, 1),
                       "ar_concurrent_us": round(ar_conc * 1e3, 1), "bucket_mib": 25,
                       "err": grp.async_error()}), flush=True)
