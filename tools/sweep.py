@@ -18,7 +18,8 @@ import torch
 import paper_conf_sigcomm_liuhlgcwz025_b200 as R
 
 N = 8
-BASE = dict(instances=18, chunkbytes=8 << 20, fifodepth=2, direct=int(os.environ.get("SWEEP_DIRECT", "1")))
+GRAPH = os.environ.get("SWEEP_GRAPH", "1") == "1"  # device-clock timing (CUDA-graph replay)
+BASE = dict(instances=14, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=int(os.environ.get("SWEEP_DIRECT", "1")))
 ELT = {"bfloat16": 2, "float32": 4, "int32": 4}
 
 
@@ -60,11 +61,28 @@ def _measure(name, coll, gopts, opts, S, dtype="bfloat16", iters=10, warm=3):
             f(s, r)
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        for _ in range(iters):
-            f(s, r)
-        e1.record()
-        torch.cuda.synchronize()
+        if GRAPH:
+            # device clock: the calls captured in one CUDA graph and replayed (an eager loop
+            # of 8 virtual-rank calls is host-bound below ~1 MiB)
+            st = torch.cuda.Stream()
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=st):
+                for _ in range(iters):
+                    f(s, r, stream=st) if coll == "allgather" else f(s, r, "sum", stream=st)
+            g.replay()
+            torch.cuda.synchronize()
+            e0.record(st)
+            with torch.cuda.stream(st):
+                g.replay()
+            e1.record(st)
+            torch.cuda.synchronize()
+            del g
+        else:
+            e0.record()
+            for _ in range(iters):
+                f(s, r)
+            e1.record()
+            torch.cuda.synchronize()
         ms = e0.elapsed_time(e1) / iters
         err = grp.async_error()
         Sb = (sn if coll != "allgather" else rn) * elt
@@ -74,7 +92,8 @@ def _measure(name, coll, gopts, opts, S, dtype="bfloat16", iters=10, warm=3):
                 "us": round(ms * 1e3, 2), "algbw_gbs": round(alg, 2), "busbw_gbs": round(bus, 2),
                 "ctas_per_rank": info["ctas"], "blocks": sum(info["blocks_per_rank"]),
                 "instances": info["instances"], "linkmodel": info["linkmodel"], "fused": info["plan"]["fused"],
-                "sched": info.get("sched"), "direct": info.get("direct"), "err": err}
+                "sched": info.get("sched"), "direct": info.get("direct"), "err": err,
+                "timing": "graph" if GRAPH else "eager"}
     finally:
         grp.destroy()
 
