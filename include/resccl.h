@@ -166,6 +166,11 @@ rescclResult_t rescclCommGetAsyncError(rescclComm_t comm, rescclResult_t* err);
  *     tbbudget=B (TBs = CTAs per rank): instances = floor(B / T_min) under the
  *     pair link model, or the port model (one duplex CTA per rank) with B instances when
  *     B < T_min or when linkmodel=port is given explicitly.
+ *     Transport and engine options: direct=0|1 (staged FIFO vs direct
+ *     push / pull, R23), pushreduce=1 (with direct: rrc operands pushed into the
+ *     receiver's FIFO, R31), sched=hpds|rr, tma=0|1, tmatile=B, tmastages=S, tmamin=B,
+ *     bulkred=-1|0|1, lookahead=0|1|2 (R30), relaybypass=0|1 (R29), devepoch=0|1,
+ *     trace=1 (TB utilisation), phase=1 (rescclGetPhaseTrace), nvls=1 (f3).
  *     t <src> <dst> <step> <chunk> <recv|rrc>
  * Environment overrides: RESCCL_INSTANCES, RESCCL_CHUNK_BYTES, RESCCL_FIFO_DEPTH,
  * RESCCL_NWARPS, RESCCL_LINK_MODEL, RESCCL_FUSE, RESCCL_TB_BUDGET.
