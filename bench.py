@@ -301,26 +301,25 @@ def main():
     # at N=1 every virtual rank's buffers share one address space, under torchrun (N>1) the
     # send and receive buffers sit in a registered symmetric window.  The lane engine's
     # cost is per TMA tile, so tiles are 24 KiB (2 stages per lane, one CTA per SM):
-    #   N=1: 14 instances x 8 virtual ranks = 112 CTAs of 256 threads (the smallest count
-    #        within noise of the best busBW, profiles/r01_ctas_nranks.jsonl: ResCCL's
-    #        point is fewer TBs), 32 MiB transfer chunks (one micro-batch
-    #        per 32 MiB algorithm chunk);
-    #   N>1: 24 CTAs of 512 threads per rank (the best per-SM geometry: 87-91 GB/s of HBM
-    #        per SM at <= 32 CTAs), 8 MiB chunks.
+    #   N=1: 12 instances x 8 virtual ranks = 96 CTAs of 384 threads (65% of the SMs; the
+    #        smallest count within 2% of the best busBW, profiles/r02_per_sm_rate.jsonl:
+    #        ResCCL's point is fewer TBs), 28 KiB tiles, 32 MiB transfer
+    #        chunks (one micro-batch per 32 MiB algorithm chunk);
+    #   N>1: 24 CTAs of 384 threads per rank, 28 KiB tiles, 8 MiB chunks.
     direct = 1 if args.direct < 0 else args.direct
     tuned = direct and not args.instances and not args.nwarps
-    inst = args.instances or ((14 if not multi else 24) if tuned else 18)
+    inst = args.instances or ((12 if not multi else 24) if tuned else 18)
     opts = {"instances": inst,
             "chunkbytes": args.chunk_bytes or ((32 << 20) if (tuned and not multi) else (8 << 20) if direct
                                                else (4 << 20)),
             "fifodepth": args.fifo_depth or 2,
-            "nwarps": args.nwarps or ((8 if not multi else 16) if tuned else None),
+            "nwarps": args.nwarps or ((12 if not multi else 12) if tuned else None),
             "tma": None if args.tma < 0 else args.tma,
             "tmastages": 2 if tuned else None,
-            # 28 KiB tiles with 16 warps: 94 GB/s of HBM per SM at 8 CTAs against 85 with 24 KiB
-            # (profiles/r02_per_sm_rate.jsonl) -- what counts at N>1, where few CTAs per rank
-            # must carry NVLink; the HBM-bound N=1 headline is equal either way (320 GB/s)
-            "tmatile": (24576 if not multi else 28672) if tuned else None,
+            # 28 KiB tiles with 12 warps (384 threads: the register cap of 16 warps, 128 per
+            # thread, spills the TMA leader loop): 95-101 GB/s of HBM per SM at 8 CTAs against
+            # 85 with 8 warps and 24 KiB tiles (profiles/r02_per_sm_rate.jsonl)
+            "tmatile": 28672 if tuned else None,
             "direct": direct, "nvls": 1 if (args.nvls and multi) else None,
             "pushreduce": 1 if (args.pushreduce and direct) else None}
     text = ir_text(R, args.algo, n, opts)

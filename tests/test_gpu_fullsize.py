@@ -23,8 +23,8 @@ from oracle import fastreplay, ir as oir, replay
 pytestmark = pytest.mark.gpu
 
 
-# bench.py's N=1 launch configuration (bench.py: instances 14 x 8 ranks = 112 CTAs)
-BENCH_OPTS = dict(instances=14, chunkbytes=32 << 20, fifodepth=2, nwarps=8, direct=1, tmastages=2, tmatile=24576)
+# bench.py's N=1 launch configuration (bench.py: instances 12 x 8 ranks = 96 CTAs of 384 threads)
+BENCH_OPTS = dict(instances=12, chunkbytes=32 << 20, fifodepth=2, nwarps=12, direct=1, tmastages=2, tmatile=28672)
 
 
 @pytest.mark.timeout(900)
