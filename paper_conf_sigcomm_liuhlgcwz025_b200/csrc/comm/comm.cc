@@ -891,6 +891,14 @@ bool host_ptr(const void* p, bool* pageable = nullptr) {
   cudaError_t e = cudaPointerGetAttributes(&at, p);
   if (e != cudaSuccess) {
     cudaGetLastError();
+    // a device address the runtime does not describe (e.g. a VMM mapping) is still device
+    // memory if the driver knows its range
+    CUdeviceptr base = 0;
+    size_t sz = 0;
+    if (driver().MemGetAddressRange(&base, &sz, (CUdeviceptr)p) == CUDA_SUCCESS && sz > 0) {
+      if (pageable) *pageable = false;
+      return false;
+    }
     fail(rescclInvalidArgument, std::string("buffer pointer not classifiable: ") + cudaGetErrorString(e));
   }
   if (pageable) *pageable = at.type == cudaMemoryTypeUnregistered;
