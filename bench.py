@@ -234,6 +234,31 @@ def cpu_fast_replay(algo: str, n: int, dtype: str, xs, count: int, threads: int,
     return S / dt * 2 * (n - 1) / n / 1e9, dt
 
 
+def cpu_per_config(cores: int, size_mb: int = 64):
+    """the oracle's C++ fast replay per BASELINE config family (8 ranks,
+    `size_mb` MiB per-rank buffer S, bf16, all host cores): busBW-equivalent GB/s."""
+    import numpy as np
+    from oracle import fastreplay, ir as oir
+    n, e = 8, 2
+    out = {}
+    for name, coll, kw in (("ring", "allreduce", {}), ("ring", "allgather", {}), ("dbt", "allreduce", {}),
+                           ("hm", "allreduce", {"g": 4}), ("synth", "allgather", {"seed": 0, "fanout": 2}),
+                           ("synth", "reducescatter", {"seed": 0, "fanout": 2})):
+        S = size_mb << 20
+        cnt = S // e if coll == "allreduce" else S // e // n      # the collective's count argument
+        xs = host_workload(n, cnt * (n if coll == "reducescatter" else 1), "bfloat16", seed=3)
+        g = oir.generate(name, coll, n, **kw)
+        outs = [np.empty(cnt * (n if coll == "allgather" else 1), np.uint16) for _ in range(n)]
+        work = [np.empty(n * cnt, np.uint16) for _ in range(n)] if coll == "reducescatter" else None
+        fastreplay.replay_full(g, xs, "bfloat16", cnt, threads=cores, outputs=outs, work=work)  # warm (pages)
+        t0 = time.perf_counter()
+        fastreplay.replay_full(g, xs, "bfloat16", cnt, threads=cores, outputs=outs, work=work)
+        dt = time.perf_counter() - t0
+        f = 2 * (n - 1) / n if coll == "allreduce" else (n - 1) / n
+        out[f"{name} {coll}"] = round(S / dt / 1e9 * f, 3)
+    return out
+
+
 def reference_impl(args):
     """--impl reference: the oracle timed on the host cores (tier framing).  A step = the
     C++ fast replay of the same workload as the ResCCL arm (same algorithm, ranks, bytes
@@ -672,6 +697,7 @@ def main():
                "python_replay": {"value": round(bus_py, 4), "unit": "GB/s", "cores": 1,
                                  "s_per_call": round(dt_py, 3), "sample": desc_py},
                "c1_replay_s": round(c1_replay_seconds(), 4),
+               "per_config_64MiB": cpu_per_config(cores),
                "c1": "BASELINE configs[0]: ring AllReduce 4096 fp32, 2 ranks, 1 TB, 4 chunks (Python replay)"}
 
     # SMs the kernel occupies: its CTAs (one or two per SM, by block size) spread over the SMs

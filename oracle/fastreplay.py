@@ -48,10 +48,11 @@ def _load():
 
 
 def replay_full(ir, inputs: List[np.ndarray], dtype: str, count: int, threads: int = 1,
-                outputs: List[np.ndarray] = None) -> List[np.ndarray]:
+                outputs: List[np.ndarray] = None, work: List[np.ndarray] = None) -> List[np.ndarray]:
     """``ir``: an oracle IR (``oracle.ir.IR``) or IR text.  ``inputs[r]``: rank r's send
     buffer.  ``outputs``: optional preallocated receive buffers (AR: may be the inputs
-    themselves, in place)."""
+    themselves, in place); ``work`` (ReduceScatter): optional preallocated N x count
+    location buffers (timing loops reuse both, so first-touch page faults stay out)."""
     lib = _load()
     text = ir if isinstance(ir, str) else ir.to_text()
     n = len(inputs)
@@ -61,7 +62,10 @@ def replay_full(ir, inputs: List[np.ndarray], dtype: str, count: int, threads: i
     if outputs is None:
         m = count * n if coll == "allgather" else count
         outputs = [np.empty(m, dtype=st) for _ in range(n)]
-    work = [np.empty(n * count, dtype=st) for _ in range(n)] if coll == "reducescatter" else None
+    if coll == "reducescatter" and work is None:
+        work = [np.empty(n * count, dtype=st) for _ in range(n)]
+    elif coll != "reducescatter":
+        work = None
     P = ctypes.c_void_p * n
     sp = P(*[x.ctypes.data for x in ins])
     rp = P(*[y.ctypes.data for y in outputs])
