@@ -40,5 +40,7 @@ def test_compute_sanitizer(tool, tma):
         pytest.skip("compute-sanitizer not available")
     rc, out = _run([cs, "--tool", tool, "--error-exitcode", "3", sys.executable, "tools/small_run.py"],
                    {"SMALL_RUN_TMA": tma}, 1250)
+    if "compute-sanitizer is closed" in out:  # the GPU pool's wrapper refuses the tool
+        pytest.skip("compute-sanitizer is closed on this GPU pool")
     assert rc == 0 and "ALL OK" in out, out[-4000:]
     assert "ERROR SUMMARY: 0 errors" in out, out[-4000:]
