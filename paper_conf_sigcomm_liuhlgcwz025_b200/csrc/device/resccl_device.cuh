@@ -165,6 +165,28 @@ __device__ __forceinline__ void fence_release() {
   jitter();
   asm volatile("fence.acq_rel" RESCCL_SC ";" ::: "memory");
 }
+// RESCCL_SPLIT_FENCE=1 (default): the one-sided fences where one side suffices.  At .gpu /
+// .sys scope the acquire half of a fence is an L1 invalidate (CCTL.IVALL): every lane
+// leader keeps its state in local memory (noinline primitives take it by reference), so
+// an invalidate after each post made the next primitive's setup re-fetch it from L2 --
+// a chain of round trips per primitive.
+//   fence_rel: orders this thread's earlier reads and writes before its later stores (the
+//     flag / credit / counter posts after a micro-batch's data moved): MEMBAR + ERRBAR, no
+//     invalidate.
+//   fence_acq: after a relaxed load observed a released value, orders it before this
+//     thread's later reads (the acquire pattern: strong read, then fence.acquire) -- in
+//     place of a second, acquiring load of the same word (one L2 round trip per handoff).
+#ifndef RESCCL_SPLIT_FENCE
+#define RESCCL_SPLIT_FENCE 1
+#endif
+__device__ __forceinline__ void fence_rel() {
+#if RESCCL_SPLIT_FENCE
+  jitter();
+  asm volatile("fence.release" RESCCL_SC ";" ::: "memory");
+#else
+  fence_release();
+#endif
+}
 __device__ __forceinline__ u64 ld_acquire(const u64* p) {
   const u64 v = ld_acquire_raw(p);
 #if RESCCL_JITTER
@@ -189,6 +211,11 @@ __device__ __forceinline__ u64 ld_relaxed(const u64* p) {
 __device__ __forceinline__ bool ready_ge(const u64* p, u64 target) {
 #if RESCCL_POLL_ACQ
   return ld_acquire(p) >= target;
+#elif RESCCL_SPLIT_FENCE
+  if (ld_relaxed(p) < target) return false;
+  asm volatile("fence.acquire" RESCCL_SC ";" ::: "memory");
+  jitter();
+  return true;
 #else
   if (ld_relaxed(p) < target) return false;
   (void)ld_acquire(p);
@@ -626,6 +653,7 @@ struct Lane {
   int pidx;                  // index of the running primitive in the rank's descriptor table
   u64* ph;                   // RESCCL_PHASE: this lane's record area (null: off)
   u32 nph;                   // RESCCL_PHASE: records written
+  u64 t_run;                 // RESCCL_PHASE: entry of the running primitive (before its setup)
   // writable lookahead (leader): the lane's push receives in lane order (descriptor index,
   // gate = 1 + lane index of the last earlier same-lane primitive a dropped implied
   // dependency pointed at), the cursor (push receive wa_c, micro-batch wa_m) of the next
@@ -936,7 +964,7 @@ __device__ __forceinline__ void post_mb(const KArgs& a, const PrimDesc& d, const
   const u64 mb_base = a.mb_base;
   const u64 in_seq = (u64)d.in_n * mb_base + (u64)d.in_pos * a.n_mb + j;
   const u64 out_seq = (u64)d.out_n * mb_base + (u64)d.out_pos * a.n_mb + j;
-  fence_release();
+  fence_rel();
   if (F & kSend) st_relaxed(p.out_flag + (out_seq % RESCCL_K), out_seq + 1);   // payload / written / readable
   if (Kind<F>::has_b) st_relaxed(p.in_cred, in_seq + 1);                        // consumed / read (push: posted earlier)
   if (d.ctr >= 0) st_relaxed(p.ctr, mb_base + j + 1);
@@ -945,7 +973,7 @@ __device__ __forceinline__ void post_mb(const KArgs& a, const PrimDesc& d, const
 template <int F>
 __device__ __forceinline__ void post_writable(const KArgs& a, const PrimDesc& d, const PrimPtrs& p, int j) {
   const u64 in_seq = (u64)d.in_n * a.mb_base + (u64)d.in_pos * a.n_mb + j;
-  fence_release();
+  fence_rel();
   st_relaxed(p.in_cred, in_seq + 1);
 }
 
@@ -1407,7 +1435,7 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
 #endif
       post_mb<F>(a, d, p, pj);
 #if RESCCL_PHASE
-      ph_rec(L, PhPipe, pj, ph_w, ph_rdy[pj & 7], 0, ph3, ph_now());
+      ph_rec(L, PhPipe, pj, ph_w, ph_rdy[pj & 7], pj == 0 ? L.t_run : 0, ph3, ph_now());
       ph_w = ph_now();
 #endif
       ++pj;
@@ -1665,6 +1693,9 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
 
 template <class T, int OP, int F>
 __device__ __noinline__ bool run(Lane& L, const PrimDesc& d) {
+#if RESCCL_PHASE
+  L.t_run = ph_now();
+#endif
   const KArgs& a = *L.a;
   const int c = d.chunk;
   PrimPtrs p;

@@ -198,6 +198,11 @@ def main():
                    "exit_after_last_post_us": round(a["exit_after_last_post_ns"] / 1e3, 2),
                    "per_kind": per_kind(lanes, plan), "path": a["path"]}
             print(json.dumps(out), flush=True)
+            if os.environ.get("PHASE_RAW"):  # every lane of instance 0, for offline timelines
+                kinds = [[pm["kind"] for pm in rp["prims"]] for rp in plan["ranks"]]
+                with open(os.environ["PHASE_RAW"], "a") as f:
+                    f.write(json.dumps({"bytes": S, "opts": OPTS, "algo": ALGO, "kinds": kinds,
+                                        "lanes": [L for L in lanes if L["inst"] == 0]}) + "\n")
         finally:
             grp.destroy()
 
