@@ -654,6 +654,7 @@ struct Lane {
   u64* ph;                   // RESCCL_PHASE: this lane's record area (null: off)
   u32 nph;                   // RESCCL_PHASE: records written
   u64 t_run;                 // RESCCL_PHASE: entry of the running primitive (before its setup)
+  u64 t_call;                // RESCCL_PHASE: the generated code reached the primitive's call
   // writable lookahead (leader): the lane's push receives in lane order (descriptor index,
   // gate = 1 + lane index of the last earlier same-lane primitive a dropped implied
   // dependency pointed at), the cursor (push receive wa_c, micro-batch wa_m) of the next
@@ -759,6 +760,8 @@ __device__ __forceinline__ void ph_rec(Lane& L, int kind, int j, u64 t0, u64 t1,
   r[3] = t2;
   r[4] = t3;
   r[5] = t4;
+  r[6] = L.t_call;
+  r[7] = L.t_run;
 #else
   (void)L; (void)kind; (void)j; (void)t0; (void)t1; (void)t2; (void)t3; (void)t4;
 #endif
@@ -770,6 +773,12 @@ __device__ __forceinline__ u64 ph_now() {
   return 0;
 #endif
 }
+// generated call sites stamp the moment the lane's code reaches a primitive's call
+#if RESCCL_PHASE
+#define RESCCL_PH_CALL(L) ((L).t_call = rdev::globaltimer())
+#else
+#define RESCCL_PH_CALL(L) ((void)0)
+#endif
 
 template <int COLL>
 __device__ __forceinline__ i64 chunk_len(const KArgs& a, int c) {
@@ -1688,6 +1697,37 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
     }
   }
   idle_off(L, t_idle);
+  return true;
+}
+
+// A run of consecutive dependency-free pull-sends in one lane (e.g. the full mesh's seven
+// "readable" posts of its sendbuf chunks, PAPER Fig. 16): a pull-send without dependencies
+// publishes a location no primitive of this kernel writes, so nothing has to be waited for;
+// run one by one, each cost a primitive switch and a fence (~1.3 us, §5.12c) and the last
+// peer to be told waited ~9 us.  One release fence, then every flag in program order (each
+// link's positions still increase, R26).  Leader only; the other threads have nothing to do.
+template <int F>
+__device__ __noinline__ bool run_post_group(Lane& L, const PrimDesc* descs, const int* idx, int n) {
+#if RESCCL_PHASE
+  L.t_run = ph_now();
+#endif
+  if (L.tid != 0) return true;
+  const KArgs& a = *L.a;
+  const int nmb = a.n_mb;
+  const u64 ph_w = ph_now();
+  fence_rel();
+  for (int i = 0; i < n; ++i) {
+    const PrimDesc& d = descs[idx[i]];
+    u64* const out_flag = at(a.arena[d.out_peer], d.out_flag + (i64)L.inst * RESCCL_FLAGSTRIDE);
+    for (int j = 0; j < nmb; ++j) {
+      const u64 out_seq = (u64)d.out_n * a.mb_base + (u64)d.out_pos * nmb + j;
+      st_relaxed(out_flag + (out_seq % RESCCL_K), out_seq + 1);
+#if RESCCL_PHASE
+      L.pidx = idx[i];
+      ph_rec(L, PhFlags, j, ph_w, ph_w, 0, 0, ph_now());
+#endif
+    }
+  }
   return true;
 }
 
