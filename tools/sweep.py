@@ -124,6 +124,23 @@ if "c3" in which:
     for S in (64 << 20, 256 << 20):
         emit(measure("ring", "allreduce", "", dict(chunkbytes=1 << 20, fifodepth=2, instances=2,
                                                    direct=BASE["direct"]), S))
+if "c3w" in which:
+    # the C3 budget sweep at the r02 per-SM geometry (12 warps, 28 KiB tiles), DBT under the
+    # port link model and HM 2x4 under the pair model (each one's better model, §5.13)
+    for name, g, cb, lm in (("dbt", "", 8 << 20, "port"), ("hm", "g=4", 1 << 20, None)):
+        for budget in (4, 8, 12, 16, 18):
+            o = dict(chunkbytes=cb, fifodepth=2, tbbudget=budget, nwarps=12, tmatile=28672, direct=BASE["direct"])
+            if lm:
+                o["linkmodel"] = lm
+            emit(measure(name, "allreduce", g, o, 256 << 20))
+if "c4w" in which:
+    # synthesized AG / RS at 256 MiB: instances x transfer chunk at 12 warps, 28 KiB tiles
+    for coll in ("allgather", "reducescatter"):
+        for inst in (3, 4):
+            for cb in (2 << 20, 8 << 20):
+                emit(measure("synth", coll, "seed=0 fanout=2", dict(instances=inst, chunkbytes=cb, fifodepth=2,
+                                                                     nwarps=12, tmatile=28672,
+                                                                     direct=BASE["direct"]), 256 << 20))
 if "c4" in which:
     for coll in ("allgather", "reducescatter"):
         for fan in (2, 3):
