@@ -655,6 +655,8 @@ struct Lane {
   u32 nph;                   // RESCCL_PHASE: records written
   u64 t_run;                 // RESCCL_PHASE: entry of the running primitive (before its setup)
   u64 t_call;                // RESCCL_PHASE: the generated code reached the primitive's call
+  u64 t_pro;                 // RESCCL_PHASE: entry of the engine function (after run's setup)
+  u64 t_end;                 // RESCCL_PHASE: the previous primitive's engine function returned
   // writable lookahead (leader): the lane's push receives in lane order (descriptor index,
   // gate = 1 + lane index of the last earlier same-lane primitive a dropped implied
   // dependency pointed at), the cursor (push receive wa_c, micro-batch wa_m) of the next
@@ -761,7 +763,10 @@ __device__ __forceinline__ void ph_rec(Lane& L, int kind, int j, u64 t0, u64 t1,
   r[4] = t3;
   r[5] = t4;
   r[6] = L.t_call;
-  r[7] = L.t_run;
+  // ns deltas, 16 bits each (saturating): run entry - call, engine entry - run entry,
+  // call - previous primitive's return
+  auto d16 = [](u64 a, u64 b) -> u64 { return (a && b && a >= b) ? (a - b > 65535 ? 65535 : a - b) : 65535; };
+  r[7] = d16(L.t_run, L.t_call) | (d16(L.t_pro, L.t_run) << 16) | (d16(L.t_call, L.t_end) << 32);
 #else
   (void)L; (void)kind; (void)j; (void)t0; (void)t1; (void)t2; (void)t3; (void)t4;
 #endif
@@ -1160,6 +1165,9 @@ __device__ __forceinline__ u32 mb_tiles(const KArgs& a, i64 len, int j, int inst
 // carries over from the plan check).
 template <class T, int OP, int F, bool BRED>
 __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
+#if RESCCL_PHASE
+  L.t_pro = ph_now();
+#endif
   const KArgs& a = *L.a;
   // Everything the loop reads per tile lives in registers: the lane, the arguments and
   // the pointers are memory-resident (their addresses are taken), and every asm
@@ -1515,6 +1523,9 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
   idle_off(L, t_idle);
   L.tseq = k0 + issued;
   L.cpar = Lcpar;
+#if RESCCL_PHASE
+  L.t_end = ph_now();
+#endif
   return true;
 }
 
@@ -1616,6 +1627,9 @@ __device__ __noinline__ bool pipe_compute(Lane& L, const PrimDesc& d, const Prim
 // posts "readable" for the next hop, which pulls from our location).
 template <int F>
 __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtrs& p) {
+#if RESCCL_PHASE
+  L.t_pro = ph_now();
+#endif
   const KArgs& a = *L.a;
   const int nmb = a.n_mb;
   const u64 mb_base = a.mb_base;
@@ -1697,6 +1711,9 @@ __device__ __noinline__ bool run_flags(Lane& L, const PrimDesc& d, const PrimPtr
     }
   }
   idle_off(L, t_idle);
+#if RESCCL_PHASE
+  L.t_end = ph_now();
+#endif
   return true;
 }
 

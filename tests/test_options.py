@@ -33,3 +33,46 @@ def test_kernel_variants_build(opts):
 def test_generated_source_uses_device_epochs():
     src = R.rescclCodegenIr(R.rescclGenerateIr("ring", "allreduce", 2), "instances=1")
     assert "epochs_begin" in src and "epochs_end" in src
+
+
+@pytest.mark.parametrize("opts", ["splitfence=0", "splitfence=1", "postgroup=0", "postgroup=1 direct=1"])
+def test_fence_and_post_group_variants_build(opts):
+    """both fence variants and both post forms compile for sm_100a."""
+    text = R.rescclGenerateIr("hm", "allreduce", 8, "g=8")
+    assert R.rescclCompileIr(text, opts + " linkmodel=port instances=1", R.rescclBfloat16, R.rescclSum) > 0
+
+
+def _calls(src):
+    import re
+    single = [int(m) for m in re.findall(r"L\.pidx = (\d+);[^\n]*rdev::run<", src)]
+    groups = [[int(x) for x in g.split(",")] for g in re.findall(r"static __constant__ int kPg\[\d+\] = \{([^}]*)\}", src)]
+    return single, groups
+
+
+def test_post_group_covers_every_primitive_once():
+    """The full mesh's send lane starts with N-1 dependency-free pull-sends: with postgroup=1
+    they become one grouped call, and every primitive of the plan is still called exactly
+    once per lane (no primitive dropped or duplicated); postgroup=0 or the ring (one pull-send
+    per lane) emit no group."""
+    text = R.rescclGenerateIr("hm", "allreduce", 8, "g=8")
+    opts = "linkmodel=port instances=1 direct=1"
+    plan = R.rescclPlanIr(text, opts)["plan"]
+    for pg in (1, 0):
+        src = R.rescclCodegenIr(text, opts + f" postgroup={pg}")
+        single, groups = _calls(src)
+        if pg:
+            assert len(groups) == 8 and all(len(g) == 7 for g in groups)
+            for r, g in enumerate(groups):
+                assert all(plan["ranks"][r]["prims"][k]["kind"] == "psend" for k in g)
+        else:
+            assert not groups
+        total = len(single) + sum(len(g) for g in groups)
+        assert total == sum(len(rp["prims"]) for rp in plan["ranks"])
+    ring = R.rescclCodegenIr(R.rescclGenerateIr("ring", "allreduce", 8), "instances=1 direct=1")
+    assert "run_post_group" not in ring
+
+
+def test_split_fence_macro():
+    text = R.rescclGenerateIr("ring", "allreduce", 4)
+    assert "#define RESCCL_SPLIT_FENCE 1" in R.rescclCodegenIr(text, "")
+    assert "#define RESCCL_SPLIT_FENCE 0" in R.rescclCodegenIr(text, "splitfence=0")

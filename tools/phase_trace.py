@@ -41,7 +41,8 @@ def decode(words):
             for k in range(1, int(hdr[2]) + 1):
                 r = words[off + 8 * k: off + 8 * k + 8]
                 recs.append({"prim": r[0] >> 32, "mb": (r[0] >> 8) & 0xFFFFFF, "kind": r[0] & 0xFF,
-                             "t": list(r[1:6]), "tc": r[6], "tr": r[7]})
+                             "t": list(r[1:6]), "tc": r[6], "d_run": r[7] & 0xFFFF, "d_pro": (r[7] >> 16) & 0xFFFF,
+                             "d_ret": (r[7] >> 32) & 0xFFFF})
             lanes.append({"block": b, "lane": ln, "entry": hdr[0], "exit": hdr[1], "rank": hdr[3],
                           "cta": hdr[4], "inst": hdr[5], "recs": recs})
     return lanes
