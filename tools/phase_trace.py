@@ -140,6 +140,24 @@ def per_kind(lanes, plan):
                 "data_med_ns": statistics.median(v["data"]) if v["data"] else None} for k, v in out.items()}
 
 
+def _graph_us(grp, s, r):
+    import torch
+    st = torch.cuda.Stream()
+    gph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(gph, stream=st):
+        grp.allreduce(s, r, stream=st)
+    for _ in range(3):
+        gph.replay()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(20):
+        gph.replay()
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) * 1e3 / 20
+
+
 def main():
     sizes = [int(x) for x in sys.argv[1:]] or [1024, 1 << 20, 16 << 20]
     text = R.rescclGenerateIr(ALGO, "allreduce", N, GOPTS)
@@ -165,20 +183,12 @@ def main():
             host_us = (_t.perf_counter() - h0) / 20 * 1e6
             torch.cuda.synchronize()
             loop_us = e0.elapsed_time(e1) * 1e3 / 20
-            # (b) the same call captured in a CUDA graph: GPU time per call
-            st = torch.cuda.Stream()
-            gph = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(gph, stream=st):
-                grp.allreduce(s, r, stream=st)
-            for _ in range(3):
-                gph.replay()
-            torch.cuda.synchronize()
-            e0.record()
-            for _ in range(20):
-                gph.replay()
-            e1.record()
-            torch.cuda.synchronize()
-            graph_us = e0.elapsed_time(e1) * 1e3 / 20
+            # (b) the same call captured in a CUDA graph: GPU time per call (needs device-side
+            # epochs: PHASE_NOGRAPH=1 skips it for devepoch=0 runs)
+            if os.environ.get("PHASE_NOGRAPH") == "1":
+                graph_us = float("nan")
+            else:
+                graph_us = _graph_us(grp, s, r)
             # (c) one traced call (the analysed one)
             e0.record()
             grp.allreduce(s, r)
