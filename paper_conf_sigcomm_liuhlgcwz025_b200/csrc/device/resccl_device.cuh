@@ -1456,10 +1456,9 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       ph_w = ph_now();
 #endif
       ++pj;
-      if (pj < nmb) {
-        T_p = mb_tiles_m<F>(aM, aMi, plen, pj, Linst, T::kSize, lo_p, nb_p, bred);
-        gp_end += T_p;
-      }
+      if (pj == nmb) break;  // all posted: the code after the loop returns the stages
+      T_p = mb_tiles_m<F>(aM, aMi, plen, pj, Linst, T::kSize, lo_p, nb_p, bred);
+      gp_end += T_p;
       prog = true;
     }
 #if !RESCCL_RING
