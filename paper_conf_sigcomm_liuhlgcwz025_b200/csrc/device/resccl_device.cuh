@@ -165,17 +165,16 @@ __device__ __forceinline__ void fence_release() {
   jitter();
   asm volatile("fence.acq_rel" RESCCL_SC ";" ::: "memory");
 }
-// RESCCL_SPLIT_FENCE=1 (default): the one-sided fences where one side suffices.  At .gpu /
-// .sys scope the acquire half of a fence is an L1 invalidate (CCTL.IVALL): every lane
-// leader keeps its state in local memory (noinline primitives take it by reference), so
-// an invalidate after each post made the next primitive's setup re-fetch it from L2 --
-// a chain of round trips per primitive.
+// RESCCL_SPLIT_FENCE=1 (default): one-sided fences where one side suffices.  At .gpu / .sys
+// scope the acquire half of a fence compiles to an L1 invalidate (CCTL.IVALL).
 //   fence_rel: orders this thread's earlier reads and writes before its later stores (the
 //     flag / credit / counter posts after a micro-batch's data moved): MEMBAR + ERRBAR, no
 //     invalidate.
-//   fence_acq: after a relaxed load observed a released value, orders it before this
-//     thread's later reads (the acquire pattern: strong read, then fence.acquire) -- in
-//     place of a second, acquiring load of the same word (one L2 round trip per handoff).
+//   ready_ge: after a relaxed load observed a released value, fence.acquire orders it before
+//     this thread's later reads (the PTX acquire pattern: strong read, then fence.acquire)
+//     in place of a second, acquiring load of the same word.
+// Both are the minimal orderings the protocol needs; on the device clock they measure the
+// same as the two-sided forms (the per-primitive cost is not a cache effect).
 #ifndef RESCCL_SPLIT_FENCE
 #define RESCCL_SPLIT_FENCE 1
 #endif
