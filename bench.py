@@ -65,7 +65,7 @@ def parse():
     p.add_argument("--inplace-steps", type=int, default=10,
                    help="also time in-place calls (recv = send) -> config.inplace_busbw_gbs")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--tuned-sweep", default="0.0009765625,0.0625,1,4,16,64,256",
+    p.add_argument("--tuned-sweep", default="0.0009765625,0.0625,0.25,1,4,16,64,256",
                    help="MiB-per-rank sizes for the size-tuned AllReduce (mesh / mesh-port schedules selected "
                         "by minbytes / maxbytes); '' = none")
     p.add_argument("--sweep", default="0.0009765625,1,16,64",
@@ -551,12 +551,22 @@ def main():
     if args.tuned_sweep and args.algo == "ring":
         two = 2 << 20
         mesh = f"g={n}"  # the hierarchical mesh at one node of all n ranks: a full mesh
-        i_big, i_mid = (14, 18) if not multi else (24, 24)
+        # r02 late (profiles/r02_lat_classes.jsonl, r02_lat_midgeo.jsonl): the 2x4 hierarchical
+        # schedule (HM g=4, pair model, 4 instances) wins from 512 KiB to 8 MiB (1 MiB 52 us,
+        # 4 MiB 72 us against the mesh's 56 / 95), 16 mesh instances beat 14 above 32 MiB
+        i_big, i_mid = (16, 18) if not multi else (24, 24)
+        small = 256 << 10
         tuned_table = [("hm", mesh, dict(instances=i_big, chunkbytes=8 << 20, linkmodel="port",
                                          minbytes=(32 << 20) + 1)),
-                       ("hm", mesh, dict(instances=i_mid, chunkbytes=8 << 20, linkmodel="port", minbytes=two + 1,
-                                         maxbytes=32 << 20)),
-                       ("hm", mesh, dict(instances=2, chunkbytes=two, maxbytes=two))]
+                       ("hm", mesh, dict(instances=i_mid, chunkbytes=8 << 20, linkmodel="port",
+                                         minbytes=(8 << 20) + 1, maxbytes=32 << 20))]
+        if n % 4 == 0 and n > 4 and not multi:
+            tuned_table.append(("hm", "g=4", dict(instances=4, chunkbytes=512 << 10, minbytes=small + 1,
+                                                  maxbytes=8 << 20)))
+        else:  # (N > 1 keeps the round-2 classes: mesh to 2 MiB, mesh under the port model above)
+            small = two
+            tuned_table[-1][2]["minbytes"] = small + 1
+        tuned_table.append(("hm", mesh, dict(instances=2, chunkbytes=two, maxbytes=small)))
         if multi:
             tcomm = R.init_process_group_comm(rank, world, local)
             tcomms = [tcomm]

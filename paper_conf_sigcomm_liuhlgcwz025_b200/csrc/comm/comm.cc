@@ -160,6 +160,7 @@ struct Options {
   int bulkred = -1;  // in-place reduce primitives: cp.reduce.async.bulk of the incoming tile
                      // (-1 = auto: on for AllReduce, where it measured +16% per SM; r01_bulkred_inplace)
   int cpoll = 0;     // combine warps: one polling warp + named barrier (1) vs all polling (0)
+  int early_exit = 1;  // the lane engine leaves its loop right after the last post
   int post_group = 1;  // consecutive dependency-free pull-sends posted as one group
   int split_fence = 1;  // one-sided release / acquire fences
   int store_lag = 1; // bulk stores a lane lets drain before it blocks to reuse a stage
@@ -224,6 +225,7 @@ void apply_kv(Options& o, const std::string& k, const std::string& v) {
   else if (k == "storelag") o.store_lag = (int)to_long(v, k);
   else if (k == "splitfence") o.split_fence = (int)to_long(v, k);
   else if (k == "postgroup") o.post_group = (int)to_long(v, k);
+  else if (k == "earlyexit") o.early_exit = (int)to_long(v, k);
   else if (k == "ring") o.ring = (int)to_long(v, k);
   else if (k == "cpoll") o.cpoll = (int)to_long(v, k);
   else if (k == "bulkred") o.bulkred = (int)to_long(v, k);
@@ -253,7 +255,7 @@ Options make_options(const Ir& ir, const char* extra) {
       {"RESCCL_INSTANCES", "instances"}, {"RESCCL_CHUNK_BYTES", "chunkbytes"}, {"RESCCL_FIFO_DEPTH", "fifodepth"},
       {"RESCCL_NWARPS", "nwarps"},       {"RESCCL_LINK_MODEL", "linkmodel"},   {"RESCCL_FUSE", "fuse"},
       {"RESCCL_TB_BUDGET", "tbbudget"}, {"RESCCL_TMA", "tma"}, {"RESCCL_TMA_TILE", "tmatile"},
-      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_POLL_ACQ", "pollacq"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_SPLIT_FENCE", "splitfence"}, {"RESCCL_POST_GROUP", "postgroup"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_BULKRED", "bulkred"}, {"RESCCL_DEVEPOCH", "devepoch"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
+      {"RESCCL_TMA_STAGES", "tmastages"}, {"RESCCL_TRACE", "trace"}, {"RESCCL_L2HINT", "l2hint"}, {"RESCCL_PREFETCH", "prefetch"}, {"RESCCL_SCHED", "sched"}, {"RESCCL_TMA_MIN", "tmamin"}, {"RESCCL_DIRECT", "direct"}, {"RESCCL_BACKOFF", "backoff"}, {"RESCCL_POLL_ACQ", "pollacq"}, {"RESCCL_JITTER", "jitter"}, {"RESCCL_RING", "ring"}, {"RESCCL_STORE_LAG", "storelag"}, {"RESCCL_SPLIT_FENCE", "splitfence"}, {"RESCCL_POST_GROUP", "postgroup"}, {"RESCCL_EARLY_EXIT", "earlyexit"}, {"RESCCL_NVLS", "nvls"}, {"RESCCL_CPOLL", "cpoll"}, {"RESCCL_BULKRED", "bulkred"}, {"RESCCL_DEVEPOCH", "devepoch"}, {"RESCCL_NVLS_CTAS", "nvlsctas"}};
   for (auto& e : envs)
     if (const char* v = getenv(e.first)) apply_kv(o, e.second, v);
   for (auto& kv : parse_kv(extra)) apply_kv(o, kv.first, kv.second);
@@ -579,6 +581,7 @@ CodegenOpts codegen_opts(const Options& o) {
   co.store_lag = o.store_lag;
   co.split_fence = o.split_fence;
   co.post_group = o.post_group;
+  co.early_exit = o.early_exit;
   co.ring = o.ring;
   co.cpoll = o.cpoll;
   co.bulkred = o.bulkred;

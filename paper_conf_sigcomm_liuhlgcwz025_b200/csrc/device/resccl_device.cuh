@@ -1116,6 +1116,10 @@ __device__ __noinline__ bool run_sync(Lane& L, const PrimDesc& d, const PrimPtrs
 #ifndef RESCCL_STORE_LAG
 #define RESCCL_STORE_LAG 1
 #endif
+// RESCCL_EARLY_EXIT=1 (default): the leader leaves its event loop right after the last post
+#ifndef RESCCL_EARLY_EXIT
+#define RESCCL_EARLY_EXIT 1
+#endif
 // parity of a quiescent mbarrier's current (incomplete) phase: the preceding phase, of
 // the other parity, tests complete
 __device__ __forceinline__ u32 mbar_phase(u32 bar) { return mbar_test(bar, 0) ? 1u : 0u; }
@@ -1455,9 +1459,15 @@ __device__ __noinline__ bool pipe_leader(Lane& L, const PrimDesc& d, const PrimP
       ph_w = ph_now();
 #endif
       ++pj;
+#if RESCCL_EARLY_EXIT
       if (pj == nmb) break;  // all posted: the code after the loop returns the stages
-      T_p = mb_tiles_m<F>(aM, aMi, plen, pj, Linst, T::kSize, lo_p, nb_p, bred);
-      gp_end += T_p;
+#else
+      if (pj < nmb)
+#endif
+      {
+        T_p = mb_tiles_m<F>(aM, aMi, plen, pj, Linst, T::kSize, lo_p, nb_p, bred);
+        gp_end += T_p;
+      }
       prog = true;
     }
 #if !RESCCL_RING

@@ -65,6 +65,7 @@ struct CodegenOpts {
   int ring = 0;                  // lane-private stage rings instead of the shared CTA pool
   int bulkred = 0;               // in-place reduces: bulk-add the incoming tile in L2
   int cpoll = 0;                 // combine warps: 1 = one polling warp + named barrier
+  int early_exit = 1;            // the lane engine leaves its loop right after the last post
   int post_group = 1;            // consecutive dependency-free pull-sends posted as one group
   int split_fence = 1;           // one-sided release / acquire fences
   int store_lag = 1;             // bulk stores a lane lets drain before it blocks to reuse a stage
