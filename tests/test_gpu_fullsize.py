@@ -78,6 +78,13 @@ def test_fullsize_elementwise(inplace):
     ("hm", "allreduce", {"g": 4}, 64, "bfloat16", dict(instances=4, chunkbytes=1 << 20, fifodepth=2)),
     ("dbt", "allreduce", {}, 256, "bfloat16", dict(instances=2, chunkbytes=4 << 20, direct=1)),
     ("dbt", "allreduce", {}, 64, "float16", dict(instances=4, chunkbytes=1 << 20, fifodepth=2)),
+    # the size-tuned classes bench.py selects: 2x4 hierarchical at 4 MiB, the
+    # full mesh under the port model at 16 MiB (18 instances) and 256 MiB (16 instances)
+    ("hm", "allreduce", {"g": 4}, 4, "bfloat16", dict(instances=4, chunkbytes=512 << 10, nwarps=8, direct=1)),
+    ("hm", "allreduce", {"g": 8}, 16, "bfloat16", dict(instances=18, chunkbytes=8 << 20, nwarps=8,
+                                                       linkmodel="port", direct=1)),
+    ("hm", "allreduce", {"g": 8}, 256, "bfloat16", dict(instances=16, chunkbytes=8 << 20, nwarps=8,
+                                                        linkmodel="port", direct=1)),
     # C4: synthesized AllGather / ReduceScatter (total buffer sizes)
     ("synth", "reducescatter", {"seed": 0, "fanout": 2}, 256, "float32", dict(instances=4, chunkbytes=1 << 20)),
     ("synth", "allgather", {"seed": 1, "fanout": 3}, 256, "bfloat16", dict(instances=3, chunkbytes=4 << 20, direct=1)),
