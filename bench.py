@@ -65,7 +65,7 @@ def parse():
     p.add_argument("--inplace-steps", type=int, default=10,
                    help="also time in-place calls (recv = send) -> config.inplace_busbw_gbs")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--tuned-sweep", default="0.0009765625,0.0625,0.25,1,4,16,64,256",
+    p.add_argument("--tuned-sweep", default="0.0009765625,0.015625,0.0625,0.25,1,4,16,64,256",
                    help="MiB-per-rank sizes for the size-tuned AllReduce (mesh / mesh-port schedules selected "
                         "by minbytes / maxbytes); '' = none")
     p.add_argument("--sweep", default="0.0009765625,1,16,64",
@@ -561,12 +561,18 @@ def main():
                        ("hm", mesh, dict(instances=i_mid, chunkbytes=8 << 20, linkmodel="port",
                                          minbytes=(8 << 20) + 1, maxbytes=32 << 20))]
         if n % 4 == 0 and n > 4 and not multi:
-            tuned_table.append(("hm", "g=4", dict(instances=4, chunkbytes=512 << 10, minbytes=small + 1,
+            # small messages (profiles/r02_lat_small*.jsonl): 128-thread CTAs; the mesh to 32 KiB
+            # (1 KiB 27 us), the 2x4 schedule above (128 KiB 29 us, 1 MiB 49 us)
+            small = 32 << 10
+            tuned_table.append(("hm", "g=4", dict(instances=4, chunkbytes=512 << 10, minbytes=two + 1,
                                                   maxbytes=8 << 20)))
+            tuned_table.append(("hm", "g=4", dict(instances=4, chunkbytes=512 << 10, nwarps=4, minbytes=small + 1,
+                                                  maxbytes=two)))
+            tuned_table.append(("hm", mesh, dict(instances=1, chunkbytes=32 << 20, nwarps=4, maxbytes=small)))
         else:  # (N > 1 keeps the round-2 classes: mesh to 2 MiB, mesh under the port model above)
             small = two
             tuned_table[-1][2]["minbytes"] = small + 1
-        tuned_table.append(("hm", mesh, dict(instances=2, chunkbytes=two, maxbytes=small)))
+            tuned_table.append(("hm", mesh, dict(instances=2, chunkbytes=two, maxbytes=small)))
         if multi:
             tcomm = R.init_process_group_comm(rank, world, local)
             tcomms = [tcomm]

@@ -166,6 +166,8 @@ rescclResult_t rescclCommGetAsyncError(rescclComm_t comm, rescclResult_t* err);
  *     tbbudget=B (TBs = CTAs per rank): instances = floor(B / T_min) under the
  *     pair link model, or the port model (one duplex CTA per rank) with B instances when
  *     B < T_min or when linkmodel=port is given explicitly.
+ *     nwarps=2 (one warp per lane) always takes the register path: the TMA lane engine
+ *     needs combine warps beside each lane's leader warp.
  *     Transport and engine options: direct=0|1 (staged FIFO vs direct
  *     push / pull, R23), pushreduce=1 (with direct: rrc operands pushed into the
  *     receiver's FIFO, R31), sched=hpds|rr, tma=0|1, tmatile=B, tmastages=S, tmamin=B,

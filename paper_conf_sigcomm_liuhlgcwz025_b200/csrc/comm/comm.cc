@@ -263,6 +263,9 @@ Options make_options(const Ir& ir, const char* extra) {
   if (o.fifo_depth < 1 || o.fifo_depth > 64) fail(rescclInvalidArgument, "fifodepth must be 1..64");
   if (o.chunk_bytes < 256 || o.chunk_bytes > (1ll << 30)) fail(rescclInvalidArgument, "chunkbytes out of range");
   if (o.nwarps < 2 || o.nwarps > 32 || o.nwarps % 2) fail(rescclInvalidArgument, "nwarps must be even, 2..32");
+  // the TMA lane engine needs combine warps beside each lane's leader warp: a one-warp lane
+  // (nwarps=2, the smallest CTAs, for small messages) always takes the register path
+  if (o.nwarps < 4) o.tma = 0;
   if (o.tma_tile < 1024 || o.tma_tile % 128 || o.tma_stages < 1 || o.tma_stages > 8 ||
       4 * o.tma_tile * o.tma_stages > 224 * 1024)
     fail(rescclInvalidArgument, "tmatile must be a multiple of 128 >= 1024, tmastages 1..8, 4*tile*stages <= 224 KiB");

@@ -42,3 +42,24 @@ def test_engine_variants_bit_exact(variant, name, kw, model, count, dtype, inpla
     exp = _expect(g, xs, dtype, count, cb, 2, model)
     for r in range(n):
         assert np.array_equal(outs[r].view(np.uint8), exp[r].view(np.uint8)), f"rank {r}"
+
+
+@pytest.mark.timeout(600)
+@pytest.mark.parametrize("name,kw,nwarps,inst,cb", [("hm", {"g": 8}, 2, 1, 32 << 20), ("hm", {"g": 8}, 4, 1, 32 << 20),
+                                                    ("hm", {"g": 4}, 4, 4, 512 << 10)])
+@pytest.mark.parametrize("count", [3 * 4096 + 77, 131072 + 11, (1 << 20) + 4099])
+def test_small_cta_geometries_bit_exact(name, kw, nwarps, inst, cb, count):
+    """The small-message classes of the size-tuned selection: 64- and 128-thread
+    CTAs.  A one-warp lane (nwarps=2) takes the register path even where slices would select
+    the TMA engine (which needs combine warps)."""
+    import paper_conf_sigcomm_liuhlgcwz025_b200 as R
+    n = 8
+    g = oir.generate(name, "allreduce", n, **kw)
+    for k, v in dict(chunkbytes=cb, instances=inst, fifodepth=2, direct=1, nwarps=nwarps).items():
+        g.extra[k] = str(v)
+    xs = inp.all_inputs("bfloat16", 33, n, count)
+    outs, info, err = run_virtual(R, g.to_text(), "allreduce", xs, "bfloat16", count)
+    assert err == 0 and info["tma"] == (0 if nwarps < 4 else 1)
+    exp = _expect(g, xs, "bfloat16", count, cb, inst, "pair")
+    for r in range(n):
+        assert np.array_equal(outs[r].view(np.uint8), exp[r].view(np.uint8)), f"rank {r}"

@@ -76,3 +76,11 @@ def test_split_fence_macro():
     text = R.rescclGenerateIr("ring", "allreduce", 4)
     assert "#define RESCCL_SPLIT_FENCE 1" in R.rescclCodegenIr(text, "")
     assert "#define RESCCL_SPLIT_FENCE 0" in R.rescclCodegenIr(text, "splitfence=0")
+
+
+def test_one_warp_lanes_take_the_register_path():
+    """nwarps=2 leaves no combine warp beside a lane's leader: the TMA engine is switched off
+    (its 'combined' barriers would count zero arrivals and never complete)."""
+    text = R.rescclGenerateIr("hm", "allreduce", 8, "g=8")
+    assert R.rescclPlanIr(text, "nwarps=2 instances=1")["tma"] == 0
+    assert R.rescclPlanIr(text, "nwarps=4 instances=1")["tma"] == 1
