@@ -554,17 +554,21 @@ def main():
         # r02 late (profiles/r02_lat_classes.jsonl, r02_lat_midgeo.jsonl): the 2x4 hierarchical
         # schedule (HM g=4, pair model, 4 instances) wins from 512 KiB to 8 MiB (1 MiB 52 us,
         # 4 MiB 72 us against the mesh's 56 / 95), 16 mesh instances beat 14 above 32 MiB
+        # warp counts (profiles/r02_lat_warps_*.jsonl, r02_lat_ab_classes.jsonl): 18 port-model
+        # instances of 128-thread CTAs to 32 MiB (16 MiB 118 us, 32 MiB 182 us on two boxes);
+        # above, 16 instances of 256-thread CTAs (the same-box A/B winner at 64 / 256 MiB)
         i_big, i_mid = (16, 18) if not multi else (24, 24)
+        w_big, w_mid = (8, 4) if not multi else (8, 8)
         small = 256 << 10
-        tuned_table = [("hm", mesh, dict(instances=i_big, chunkbytes=8 << 20, linkmodel="port",
+        tuned_table = [("hm", mesh, dict(instances=i_big, chunkbytes=8 << 20, linkmodel="port", nwarps=w_big,
                                          minbytes=(32 << 20) + 1)),
-                       ("hm", mesh, dict(instances=i_mid, chunkbytes=8 << 20, linkmodel="port",
+                       ("hm", mesh, dict(instances=i_mid, chunkbytes=8 << 20, linkmodel="port", nwarps=w_mid,
                                          minbytes=(8 << 20) + 1, maxbytes=32 << 20))]
         if n % 4 == 0 and n > 4 and not multi:
             # small messages (profiles/r02_lat_small*.jsonl): 128-thread CTAs; the mesh to 32 KiB
             # (1 KiB 27 us), the 2x4 schedule above (128 KiB 29 us, 1 MiB 49 us)
             small = 32 << 10
-            tuned_table.append(("hm", "g=4", dict(instances=4, chunkbytes=512 << 10, minbytes=two + 1,
+            tuned_table.append(("hm", "g=4", dict(instances=4, chunkbytes=512 << 10, nwarps=6, minbytes=two + 1,
                                                   maxbytes=8 << 20)))
             tuned_table.append(("hm", "g=4", dict(instances=4, chunkbytes=512 << 10, nwarps=4, minbytes=small + 1,
                                                   maxbytes=two)))
