@@ -174,6 +174,7 @@ rescclResult_t rescclCommGetAsyncError(rescclComm_t comm, rescclResult_t* err);
  *     bulkred=-1|0|1, lookahead=0|1|2 (R30), relaybypass=0|1 (R29), devepoch=0|1,
  *     splitfence=0|1 (one-sided release / acquire fences),
  *     postgroup=0|1 (consecutive dependency-free pull-sends posted as one group),
+ *     earlyexit=0|1 (the lane engine leaves its loop right after a primitive's last post),
  *     trace=1 (TB utilisation), phase=1 (rescclGetPhaseTrace), nvls=1 (f3).
  *     t <src> <dst> <step> <chunk> <recv|rrc>
  * Environment overrides: RESCCL_INSTANCES, RESCCL_CHUNK_BYTES, RESCCL_FIFO_DEPTH,

@@ -35,7 +35,7 @@ def test_generated_source_uses_device_epochs():
     assert "epochs_begin" in src and "epochs_end" in src
 
 
-@pytest.mark.parametrize("opts", ["splitfence=0", "splitfence=1", "postgroup=0", "postgroup=1 direct=1"])
+@pytest.mark.parametrize("opts", ["splitfence=0", "splitfence=1", "postgroup=0", "postgroup=1 direct=1", "earlyexit=0"])
 def test_fence_and_post_group_variants_build(opts):
     """both fence variants and both post forms compile for sm_100a."""
     text = R.rescclGenerateIr("hm", "allreduce", 8, "g=8")
